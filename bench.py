@@ -1,0 +1,428 @@
+#!/usr/bin/env python3
+"""Benchmark: batched FP32 SPOTRF (lower, in place) on interleaved storage.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--workload c2|c1|c3|c2i|c4n<N>] [--n --batch --chunk --kind]
+
+A "step" is one pass of the hot path (addressing, load,
+pivot/sqrt, column scale, rank-1 update, store + info + fused failure count,
+tuning-table dispatch; plus the failure-count all-reduce when N > 1) over one
+batch of synthetic SPD matrices already resident in HBM: exactly one launch of
+our factorization kernel per step.  Every step factors a DIFFERENT
+pre-generated buffer (the factorization is in place), each larger than L2,
+so no step sees another's data in cache; when K exceeds the buffers that fit
+in HBM the pool is regenerated between groups of steps, outside the timed
+region.  Timing: CUDA events on the launching stream, barrier +
+synchronize on both sides, max over ranks.  Default workload: BASELINE.json
+configs[1] (n=16, batch=1M per GPU, chunk 32) -- weak scaling over GPUs.
+
+Prints ONE JSON line (rank 0).  Metric unit: Gflop/s with n^3/3 flops per
+matrix; the HBM side of the metric is in "hbm_gbs" and
+"roofline".
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+METRIC = "batched SPOTRF Gflop/s and HBM GB/s vs n (interleaved), 1/2/4/8 B200"
+
+WORKLOADS = {
+    "c2": dict(n=16, batch=1 << 20, chunk=32, kind="dd",
+               desc="BASELINE configs[1]: n=16, batch=1M (1048576) per GPU, chunked interleaved "
+                    "C=32, diagonally dominant SPD"),
+    "c2i": dict(n=16, batch=1 << 20, chunk=0, kind="dd",
+                desc="configs[1] variant: n=16, batch=1M per GPU, simple (fully) interleaved"),
+    "c1": dict(n=8, batch=16384, chunk=32, kind="dd",
+               desc="BASELINE configs[0]: n=8, batch=16384, chunk 32 (launch/latency-bound)"),
+    "c3": dict(n=32, batch=1 << 22, chunk=32, kind="als",
+               desc="BASELINE configs[2]: n=32, batch=4M, ALS-shaped regularised Gram, chunk 32"),
+}
+
+FLAG_NAMES = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+              0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+              0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+              0x100: "display_clock_setting"}
+
+
+def flops_per_matrix(n):          # "the standard formula, N^3/3"
+    return n ** 3 / 3.0
+
+
+def bytes_per_matrix(n):          # lower triangle read + written, FP32, + int32 info
+    return 4 * n * (n + 1) + 4
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="c2")
+    ap.add_argument("--n", type=int)
+    ap.add_argument("--batch", type=int)
+    ap.add_argument("--chunk", type=int)
+    ap.add_argument("--kind")
+    ap.add_argument("--tune", help='JSON tuning override, e.g. {"variant":2,"param":18,...}')
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--cpu-seconds", type=float, default=8.0,
+                    help="target CPU time of the cpu_baseline sample")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--max-pool-gb", type=float, default=120.0)
+    return ap.parse_args()
+
+
+def workload(a):
+    if a.workload.startswith("c4n"):
+        w = dict(n=int(a.workload[3:]), batch=1 << 20, chunk=32, kind="dd",
+                 desc=f"BASELINE configs[3] point: n={a.workload[3:]}, batch=1M, chunk 32")
+    else:
+        w = dict(WORKLOADS[a.workload])
+    for k in ("n", "batch", "chunk", "kind"):
+        v = getattr(a, k)
+        if v is not None:
+            w[k] = v
+            w["desc"] = w["desc"] + f" [override {k}={v}]"
+    w["name"] = a.workload
+    return w
+
+
+def host_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
+def measured_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def traffic_from_profiles(w):
+    """dram read+write bytes per launch of the factor kernel from a committed
+    ncu --set full capture summary (profiles/ncu_traffic.json), if any."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        d = json.load(open(p))
+        key = f"n{w['n']}_b{w['batch']}_c{w['chunk']}"
+        return d[key]["dram_bytes_per_launch"]
+    except Exception:
+        return None
+
+
+# --------------------------------------------------------------------- CPU side
+def cpu_oracle_rate(n, kind, target_s, max_batch, seed=2017):
+    """Time the oracle (as it stands) on a bounded sample of the workload."""
+    import numpy as np
+
+    import oracle
+    import synth
+    cores = oracle.default_threads()
+    probe = min(max_batch, max(256, int(2e6 / max(1.0, flops_per_matrix(n)))))
+    A = synth.generate(n, kind, seed, np.arange(probe, dtype=np.uint64))
+    t0 = time.perf_counter()
+    oracle.potrf(n, A, nthreads=cores)
+    dt = max(time.perf_counter() - t0, 1e-6)
+    S = int(min(max_batch, max(probe, probe * target_s / dt)))
+    total_t, done, block = 0.0, 0, 1 << 18
+    while done < S:
+        m = min(block, S - done)
+        A = synth.generate(n, kind, seed, np.arange(done, done + m, dtype=np.uint64))
+        t0 = time.perf_counter()
+        oracle.potrf(n, A, nthreads=cores)
+        total_t += time.perf_counter() - t0
+        done += m
+    gflops = S * flops_per_matrix(n) / total_t / 1e9
+    return dict(value=round(gflops, 4), unit="Gflop/s", cores=cores, kind="oracle",
+                sample=f"matrices 0..{S - 1} of the workload ({S} of {max_batch}), canonical "
+                       f"FP32 in, FP64 Algorithm 1, {cores} threads, {total_t:.2f} s; "
+                       f"generation excluded")
+
+
+def run_reference(a, w):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import numpy as np
+
+    import oracle
+    import synth
+    n, kind = w["n"], w["kind"]
+    cores = oracle.default_threads()
+    probe = min(w["batch"], 4096)
+    A = synth.generate(n, kind, 2017, np.arange(probe, dtype=np.uint64))
+    t0 = time.perf_counter()
+    oracle.potrf(n, A, nthreads=cores)
+    dt = max(time.perf_counter() - t0, 1e-6)
+    budget = 90.0 / max(1, a.steps + a.warmup)           # whole run within ~1.5 min
+    S = int(min(w["batch"], max(probe, probe * budget / dt)))
+    A = synth.generate(n, kind, 2017, np.arange(S, dtype=np.uint64))
+    for _ in range(a.warmup):
+        oracle.potrf(n, A, nthreads=cores)
+    times = []
+    for _ in range(a.steps):
+        t0 = time.perf_counter()
+        oracle.potrf(n, A, nthreads=cores)
+        times.append(time.perf_counter() - t0)
+    tot = sum(times)
+    value = S * a.steps * flops_per_matrix(n) / tot / 1e9
+    sample = (f"each step: matrices 0..{S - 1} of the workload ({S} of {w['batch']}), canonical "
+              f"FP32 in, FP64 Algorithm 1 (oracle/cholesky.c), {cores} host threads")
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "Gflop/s",
+        "n_gpus": a.gpus, "steps": a.steps, "warmup": a.warmup,
+        "ms_per_step": round(1e3 * tot / a.steps, 4), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": config_of(w, a),
+        "cpu_baseline": {"value": round(value, 4), "unit": "Gflop/s", "cores": cores,
+                         "kind": "oracle", "sample": sample},
+        "e2e": {"value": round(value, 4), "unit": "Gflop/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def config_of(w, a):
+    return {"workload": w["desc"], "n": w["n"], "batch_per_gpu": w["batch"], "chunk": w["chunk"],
+            "generator": w["kind"], "layout": "chunked interleaved" if w["chunk"] else "simple interleaved",
+            "parallelism": f"batch split over {a.gpus} GPU(s), 1 all-reduce of the failure count",
+            "l2": "inputs larger than L2 (126 MB); every step factors a distinct pre-generated buffer"}
+
+
+# --------------------------------------------------------------------- clocks
+class ClockSampler:
+    def __init__(self, index):
+        self.samples, self.reasons, self.max_mhz = [], 0, None
+        self._stop = threading.Event()
+        self._t = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _run(self):
+        nv = self.nv
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                fn = getattr(nv, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+                    nv.nvmlDeviceGetCurrentClocksThrottleReasons
+                self.reasons |= int(fn(self.h))
+            except Exception:
+                pass
+            time.sleep(0.0005)
+
+    def start(self):
+        if self.nv is not None:
+            self._stop.clear()
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+
+    def stop(self):
+        if self._t is not None:
+            self._stop.set()
+            self._t.join()
+            self._t = None
+
+    def report(self):
+        names = [v for k, v in FLAG_NAMES.items() if self.reasons & k and k != 0x1]
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": names, "samples": len(self.samples)}
+
+
+# --------------------------------------------------------------------- GPU side
+def run_ours(a, w):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_gatesklpd17_b200 as bsp
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    bsp.lib()
+
+    n, B, chunk, kind = w["n"], w["batch"], w["chunk"], w["kind"]
+    b0 = rank * B                                # disjoint global indices per rank
+    tune = json.loads(a.tune) if a.tune else None
+    tsel = bsp.bspotrf_get_tuning(n, chunk).as_dict() if tune is None else tune
+    elems = bsp.batch_interleaved_elems(n, B, chunk)
+    buf_bytes = elems * 4 + B * 4
+    free, _ = torch.cuda.mem_get_info(dev)
+    fit = int(min(a.max_pool_gb * 2**30, 0.80 * free) // buf_bytes)
+    P = max(1, min(a.steps, fit))
+    stream = torch.cuda.current_stream(dev)
+    pool = []
+    for _ in range(P):
+        A = torch.empty(elems, dtype=torch.float32, device=dev)
+        info = torch.empty(B, dtype=torch.int32, device=dev)
+        cnt = torch.zeros(1, dtype=torch.int32, device=dev)
+        pool.append((A, info, cnt))
+
+    def regen():
+        for A, _, cnt in pool:
+            bsp.bspotrf_synth_generate(n, B, chunk, A, kind=kind, seed=2017, b0=b0, stream=stream)
+            cnt.zero_()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def step(i):
+        A, info, cnt = pool[i % P]
+        bsp.batch_spotrf_interleaved_ex(n, B, chunk, A, info, nfailed=cnt, tune=tune, stream=stream)
+
+    regen()
+    for i in range(a.warmup):
+        step(i)
+        if world > 1:
+            dist.all_reduce(pool[i % P][2])
+    torch.cuda.synchronize(dev)
+    regen()
+    torch.cuda.synchronize(dev)
+
+    clk = ClockSampler(local)
+    total_ms, launch_ms, done = 0.0, [], 0
+    fails = 0
+    while done < a.steps:
+        g = min(P, a.steps - done)
+        if done > 0:
+            regen()
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+              for _ in range(g)]
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        barrier()
+        torch.cuda.synchronize(dev)
+        clk.start()
+        e0.record(stream)
+        for i in range(g):
+            ev[i][0].record(stream)
+            step(i)
+            ev[i][1].record(stream)
+            if world > 1:                      # a9: the one collective, 4 bytes
+                dist.all_reduce(pool[i][2])
+        e1.record(stream)
+        torch.cuda.synchronize(dev)
+        clk.stop()
+        barrier()
+        total_ms += e0.elapsed_time(e1)
+        launch_ms += [s.elapsed_time(t) for s, t in ev]
+        fails += sum(int(pool[i][2].item()) for i in range(g))
+        done += g
+    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+    lm = torch.tensor([statistics.mean(launch_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(lm, op=dist.ReduceOp.MAX)
+    total_ms, mean_launch_ms = float(t.item()), float(lm.item())
+    # correctness guard on the timed output (DD/ALS inputs are SPD)
+    bad = sum(int((pool[i][1] != 0).sum().item()) for i in range(min(P, a.steps)))
+    if bad or fails:
+        raise SystemExit(f"bench: {bad} nonzero info / {fails} counted failures on SPD input")
+
+    ms_per_step = total_ms / a.steps
+    value = world * B * flops_per_matrix(n) / (ms_per_step * 1e-3) / 1e9
+    alg_bytes = B * bytes_per_matrix(n)
+    achieved = alg_bytes / (mean_launch_ms * 1e-3) / 1e9
+    peak, peak_src = measured_peak()
+    hbm_gbs = world * alg_bytes / (ms_per_step * 1e-3) / 1e9
+
+    # ---------------- e2e: the host-buffer C-ABI call, copies inside the timed region
+    e2e = None
+    del pool
+    torch.cuda.empty_cache()
+    if not a.no_e2e and a.e2e_steps > 0:
+        dA = torch.empty(elems, dtype=torch.float32, device=dev)
+        bsp.bspotrf_synth_generate(n, B, chunk, dA, kind=kind, seed=2017, b0=b0, stream=stream)
+        pristine = dA.cpu()
+        del dA
+        hA = torch.empty(elems, dtype=torch.float32).pin_memory()
+        hinfo = torch.empty(B, dtype=torch.int32).pin_memory()
+        times = []
+        for s in range(a.e2e_steps + 1):
+            hA.copy_(pristine)
+            barrier()
+            t0 = time.perf_counter()
+            nf = bsp.batch_spotrf_interleaved_host(n, B, chunk, hA, hinfo, stream=stream)
+            if world > 1:
+                c = torch.tensor([nf], dtype=torch.int32, device=dev)
+                dist.all_reduce(c)
+                nf = int(c.item())
+            dt = time.perf_counter() - t0
+            if nf:
+                raise SystemExit(f"bench e2e: {nf} failures on SPD input")
+            if s > 0:                      # first call warms the pool / streams
+                times.append(dt)
+        tt = torch.tensor([sum(times) / len(times)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        hb = bsp.batch_spotrf_host_bytes(n, B, chunk)
+        e2e = {"value": round(world * B * flops_per_matrix(n) / float(tt.item()) / 1e9, 3),
+               "unit": "Gflop/s", "h2d_bytes_per_step": hb, "d2h_bytes_per_step": hb + 4 * B + 4,
+               "ms_per_step": round(float(tt.item()) * 1e3, 3),
+               "path": "batch_spotrf_interleaved_host (pinned host interleaved storage; lower "
+                       "triangle 2-D copies H2D, kernel, D2H + info, 3-stream slab pipeline)"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not a.no_cpu_baseline:
+        cpu = cpu_oracle_rate(n, kind, a.cpu_seconds, B)
+
+    line = {
+        "metric": METRIC, "value": round(value, 3), "unit": "Gflop/s", "n_gpus": world,
+        "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(ms_per_step, 5),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic (seeded counter-hash generator on device)",
+        "config": dict(config_of(w, a), tuning=tsel),
+        "hbm_gbs": round(hbm_gbs, 2),
+        "roofline": {"bound": "hbm", "achieved": round(achieved, 2), "peak": peak, "unit": "GB/s",
+                     "frac": round(achieved / peak, 4), "traffic": traffic_from_profiles(w),
+                     "peak_source": peak_src,
+                     "kernel": f"factorization kernel (variant {tsel['variant']}), "
+                               f"{bytes_per_matrix(n)} B/matrix x {B} matrices per launch, "
+                               f"mean launch {mean_launch_ms:.4f} ms"},
+        "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": a.steps,
+        "clocks": clk.report(),
+    }
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    a = parse()
+    w = workload(a)
+    if a.impl == "reference":
+        return run_reference(a, w)
+    return run_ours(a, w)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

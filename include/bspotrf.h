@@ -1,0 +1,146 @@
+/*
+ * bspotrf.h -- B200 (sm_100a) batched single-precision Cholesky factorization
+ * (SPOTRF, lower, in place) of very many tiny SPD matrices stored in the
+ * interleaved / chunked-interleaved layout of
+ *   Gates, Kurzak, Luszczek, Pei, Dongarra, "Autotuning Batch Cholesky
+ *   Factorization in CUDA with Interleaved Layout of Matrices", IPDPS-W 2017
+ *   (cited below as PAPER.md:<line>, the text of that paper).
+ *
+ * C ABI: plain pointers and sizes, no C++ or torch types.  Link with
+ * libbspotrf.so.  All "device pointers" are CUDA global-memory pointers owned
+ * by the caller; "stream" is a cudaStream_t (0 = legacy default stream).
+ *
+ * ----------------------------------------------------------------------------
+ * LAYOUT (Sec. II.B, Figs. 7-8; address formula from Fig. 10,
+ * PAPER.md:222-231; readings R6/R7 in DESIGN.md)
+ *   Every matrix is stored full n x n, column-major (lda = n); only the lower
+ *   triangle (i >= j) is read or written.  With chunk size C (C = batch when
+ *   chunk == 0, "simple interleaved", Fig. 7; otherwise C = chunk, a multiple
+ *   of 32, "chunked interleaved", Fig. 8), element (i, j) of matrix b is the
+ *   float at
+ *        A[(b / C) * C * n*n + (i + j*n) * C + (b % C)].
+ *   Storage holds ceil(batch/C)*C matrices (batch_interleaved_elems); the pad
+ *   lanes of the last chunk are never read as data and never written.
+ *
+ * ERRORS (LAPACK xerbla style): return 0 on success; -i if argument i is
+ * illegal (nothing is enqueued); a positive value is a cudaError_t from the
+ * launch.  No exceptions, no exit(), no printing.  Calls only ENQUEUE work on
+ * `stream` (except batch_spotrf_interleaved_host, which is blocking); read
+ * results after synchronising the stream.  No hidden allocation except in
+ * batch_spotrf_interleaved_host.  Thread-safe and reentrant.
+ * ----------------------------------------------------------------------------
+ */
+#ifndef BSPOTRF_H
+#define BSPOTRF_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st *bspotrf_stream_t; /* == cudaStream_t */
+
+#define BSPOTRF_MAX_N 64
+
+/* Kernel variants.  All right-looking-order variants
+ * perform the same per-element FP32 operation sequence (sqrt.rn, rcp.rn,
+ * mul.rn, fma.rn in k order), so their outputs are bitwise identical. */
+enum {
+    BSPOTRF_VARIANT_AUTO = 0, /* tuning table                                  */
+    BSPOTRF_VARIANT_REG = 1,  /* whole lower triangle in registers, n <= 24    */
+    BSPOTRF_VARIANT_SMEM = 2, /* left panel of `param` columns staged in shared
+                                 memory (TMA bulk or cp.async), trailing
+                                 triangle in registers; 2 <= n <= 32           */
+    BSPOTRF_VARIANT_TILE = 3  /* paper's top-looking tile algorithm (Figs. 9-11)
+                                 with param x param register tiles, tiles
+                                 streamed from global memory; any n <= 64      */
+};
+
+/* Launch tuning (a row of the autotuning table). */
+typedef struct {
+    int variant;           /* BSPOTRF_VARIANT_*                                */
+    int threads_per_block; /* multiple of 32, 32..1024; 0 = variant default.
+                              SMEM variant with TMA staging uses one chunk per
+                              block and ignores this.                         */
+    int param;             /* SMEM: panel width s; TILE: tile size nb; REG: 0 */
+    int staging;           /* SMEM only: 0 = auto, 1 = TMA bulk copy
+                              (cp.async.bulk, needs chunk in {32,64,128}),
+                              2 = per-thread cp.async                         */
+} bspotrf_tuning;
+
+/* Library version (major*10000 + minor*100 + patch). */
+int bspotrf_version(void);
+
+/* Number of floats the interleaved storage of `batch` n x n matrices with
+ * chunk size `chunk` occupies: ceil(batch/C)*C*n*n (C = batch if chunk == 0).
+ * Returns 0 if n == 0 or batch == 0, -1 on illegal arguments. */
+int64_t batch_interleaved_elems(int n, int64_t batch, int chunk);
+
+/* Batched SPOTRF, lower, in place (Alg. 1; Fig. 9 op order).
+ *   n      1..64 (0 -> quick return)                                  arg 1
+ *   batch  >= 0 (0 -> quick return)                                   arg 2
+ *   chunk  0 (simple interleaved) or a positive multiple of 32        arg 3
+ *   A      device, batch_interleaved_elems(n,batch,chunk) floats,
+ *          16-byte aligned; on return the lower triangle of every
+ *          matrix holds L with A = L L^T; the strict upper triangle
+ *          and pad lanes are untouched                                arg 4
+ *   info   device int32[batch]: 0 = success, k > 0 = the leading
+ *          minor of order k is not positive definite (pivot !(>0),
+ *          NaN included; LAPACK convention, reading R1).  Columns
+ *          j < k-1 of a failed matrix are final; the rest is
+ *          unspecified (R2)                                           arg 5
+ *   stream                                                            arg 6
+ * Errors: -1 n, -2 batch, -3 chunk, -4 A null/misaligned, -5 info null. */
+int batch_spotrf_interleaved(int n, int64_t batch, int chunk, float *A,
+                             int32_t *info, bspotrf_stream_t stream);
+
+/* As above, plus:
+ *   nfailed  device int32* or NULL: atomically INCREMENTED by the number of
+ *            matrices with info != 0 (the caller zeroes it) -- fused into the
+ *            factorization kernel (warp ballot + popc + one atomic per warp)
+ *   tune     NULL = tuning table; otherwise an explicit launch tuning
+ *            (-7 if the requested variant/param/staging is not available
+ *            for this n and chunk). */
+int batch_spotrf_interleaved_ex(int n, int64_t batch, int chunk, float *A,
+                                int32_t *info, int32_t *nfailed,
+                                const bspotrf_tuning *tune,
+                                bspotrf_stream_t stream);
+
+/* The tuning the table selects for (n, chunk) (chunk as in the factor call).
+ * Returns 0 and fills *out, or -1/-3 on an illegal n/chunk. */
+int bspotrf_get_tuning(int n, int chunk, bspotrf_tuning *out);
+
+/* Layout conversion, out of place, bit-exact (a pure permutation):
+ * canonical = batch consecutive n x n column-major matrices,
+ * batch*n*n floats; interleaved as above.  src and dst must not overlap.
+ * Pad lanes of the interleaved side are never read or written.
+ * Errors: -1 n, -2 batch, -3 chunk, -4 src null, -5 dst null or overlapping. */
+int batch_canonical_to_interleaved(int n, int64_t batch, int chunk,
+                                   const float *src_canonical,
+                                   float *dst_interleaved,
+                                   bspotrf_stream_t stream);
+int batch_interleaved_to_canonical(int n, int64_t batch, int chunk,
+                                   const float *src_interleaved,
+                                   float *dst_canonical,
+                                   bspotrf_stream_t stream);
+
+/* End-to-end call on HOST buffers (blocking).  hA is the interleaved storage
+ * in host memory (pinned memory gives asynchronous, overlapped copies), hinfo
+ * host int32[batch], nfailed_out host int32* or NULL (set, not incremented).
+ * Only the lower triangle of each matrix crosses PCIe: per column one 2-D copy
+ * per slab.  Slabs of `slab` matrices (rounded to whole chunks; 0 = auto) are
+ * pipelined over three streams (H2D / factor / D2H) with device workspace from
+ * the stream-ordered allocator.  `stream` orders the call after prior work.
+ * Errors as batch_spotrf_interleaved, plus -6 slab < 0; positive = CUDA error. */
+int batch_spotrf_interleaved_host(int n, int64_t batch, int chunk, float *hA,
+                                  int32_t *hinfo, int32_t *nfailed_out,
+                                  int64_t slab, bspotrf_stream_t stream);
+
+/* Bytes of A the host call moves each way (lower triangles only). */
+int64_t batch_spotrf_host_bytes(int n, int64_t batch, int chunk);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BSPOTRF_H */

@@ -1,0 +1,189 @@
+// api.cu -- the C ABI of libbspotrf (include/bspotrf.h): argument checks,
+// tuning-table lookup and dispatch to the per-(n, variant, chunk) kernel
+// instances registered in gen/registry.inc.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <mutex>
+#include <unordered_map>
+
+#include "../../include/bspotrf.h"
+#include "launch.h"
+
+namespace bsp {
+
+cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float *src, float *dst,
+                           cudaStream_t stream);
+
+struct InstEntry {
+    int variant;  // BSPOTRF_VARIANT_*
+    int n;
+    int param;    // SMEM: S; TILE: NB; REG: 0
+    int ct;       // compile-time chunk (0 = runtime stride)
+    int tma;      // SMEM staging: 1 = TMA bulk, 0 = cp.async
+    LaunchFn fn;
+};
+
+struct TuneEntry {
+    int n;
+    int chunk_class;  // 0: chunk==0 (simple interleaved), 1: chunk>0
+    bspotrf_tuning t;
+};
+
+#include "gen/registry.inc"      // kInstances[]
+#include "gen/tuning_table.inc"  // kTuning[]
+
+static inline uint64_t key_of(int variant, int n, int param, int ct, int tma) {
+    return ((uint64_t)variant << 40) | ((uint64_t)n << 32) | ((uint64_t)param << 20) |
+           ((uint64_t)ct << 4) | (uint64_t)tma;
+}
+
+static std::once_flag g_once;
+static std::unordered_map<uint64_t, LaunchFn> *g_inst = nullptr;
+
+static void init_tables() {
+    std::call_once(g_once, [] {
+        auto *m = new std::unordered_map<uint64_t, LaunchFn>();
+        for (const auto &e : kInstances) (*m)[key_of(e.variant, e.n, e.param, e.ct, e.tma)] = e.fn;
+        g_inst = m;
+    });
+}
+
+static LaunchFn find(int variant, int n, int param, int ct, int tma) {
+    auto it = g_inst->find(key_of(variant, n, param, ct, tma));
+    return it == g_inst->end() ? nullptr : it->second;
+}
+
+static bool default_tuning(int n, int chunk, bspotrf_tuning *t) {
+    for (const auto &e : kTuning) {
+        if (e.n == n && e.chunk_class == (chunk > 0 ? 1 : 0)) {
+            *t = e.t;
+            return true;
+        }
+    }
+    return false;
+}
+
+// Resolve a tuning to a launcher.  Returns nullptr if unavailable.
+static LaunchFn resolve(int n, int chunk, const bspotrf_tuning &t, int *tpb_out) {
+    const bool tmpl_chunk = chunk == 32 || chunk == 64 || chunk == 128;
+    *tpb_out = t.threads_per_block;
+    switch (t.variant) {
+    case BSPOTRF_VARIANT_REG:
+        return find(BSPOTRF_VARIANT_REG, n, 0, tmpl_chunk ? chunk : 0, 0);
+    case BSPOTRF_VARIANT_SMEM: {
+        int staging = t.staging;
+        if (staging == 0) staging = tmpl_chunk ? 1 : 2;
+        if (staging == 1) {
+            if (!tmpl_chunk) return nullptr;
+            *tpb_out = chunk;
+            return find(BSPOTRF_VARIANT_SMEM, n, t.param, chunk, 1);
+        }
+        LaunchFn f = find(BSPOTRF_VARIANT_SMEM, n, t.param, chunk == 32 ? 32 : 0, 0);
+        return f ? f : find(BSPOTRF_VARIANT_SMEM, n, t.param, 0, 0);
+    }
+    case BSPOTRF_VARIANT_TILE:
+        return find(BSPOTRF_VARIANT_TILE, n, t.param, 0, 0);
+    default:
+        return nullptr;
+    }
+}
+
+static int check_common(int n, int64_t batch, int chunk) {
+    if (n < 0 || n > BSPOTRF_MAX_N) return -1;
+    if (batch < 0) return -2;
+    if (chunk < 0 || (chunk % 32) != 0) return -3;
+    return 0;
+}
+
+}  // namespace bsp
+
+using namespace bsp;
+
+extern "C" int bspotrf_version(void) { return 10000; }
+
+extern "C" int64_t batch_interleaved_elems(int n, int64_t batch, int chunk) {
+    if (check_common(n, batch, chunk) != 0) return -1;
+    if (n == 0 || batch == 0) return 0;
+    const int64_t C = chunk > 0 ? chunk : batch;
+    return ((batch + C - 1) / C) * C * (int64_t)n * n;
+}
+
+extern "C" int bspotrf_get_tuning(int n, int chunk, bspotrf_tuning *out) {
+    const int rc = check_common(n, 1, chunk);
+    if (rc != 0) return rc;
+    if (out == nullptr) return -3;
+    if (!default_tuning(n, chunk, out)) {
+        out->variant = BSPOTRF_VARIANT_TILE;
+        out->threads_per_block = 128;
+        out->param = n <= 8 ? 4 : 8;
+        out->staging = 0;
+    }
+    return 0;
+}
+
+extern "C" int batch_spotrf_interleaved_ex(int n, int64_t batch, int chunk, float *A, int32_t *info,
+                                           int32_t *nfailed, const bspotrf_tuning *tune,
+                                           bspotrf_stream_t stream) {
+    int rc = check_common(n, batch, chunk);
+    if (rc != 0) return rc;
+    if (n == 0 || batch == 0) return 0;
+    if (A == nullptr || (reinterpret_cast<uintptr_t>(A) & 15u) != 0) return -4;
+    if (info == nullptr) return -5;
+    init_tables();
+    bspotrf_tuning t;
+    if (tune) {
+        t = *tune;
+        if (t.variant == BSPOTRF_VARIANT_AUTO) bspotrf_get_tuning(n, chunk, &t);
+        if (t.threads_per_block < 0 || t.threads_per_block > 1024 || (t.threads_per_block % 32) != 0)
+            return -7;
+    } else {
+        bspotrf_get_tuning(n, chunk, &t);
+    }
+    int tpb = 0;
+    LaunchFn fn = resolve(n, chunk, t, &tpb);
+    if (fn == nullptr) return -7;
+    FactorArgs a;
+    a.A = A;
+    a.info = info;
+    a.nfailed = nfailed;
+    a.batch = batch;
+    a.cstride = chunk > 0 ? chunk : batch;
+    a.tpb = tpb;
+    a.stream = (cudaStream_t)stream;
+    const cudaError_t e = fn(a);
+    return e == cudaSuccess ? 0 : (int)e;
+}
+
+extern "C" int batch_spotrf_interleaved(int n, int64_t batch, int chunk, float *A, int32_t *info,
+                                        bspotrf_stream_t stream) {
+    return batch_spotrf_interleaved_ex(n, batch, chunk, A, info, nullptr, nullptr, stream);
+}
+
+static int convert_common(int dir, int n, int64_t batch, int chunk, const float *src, float *dst,
+                          bspotrf_stream_t stream) {
+    int rc = check_common(n, batch, chunk);
+    if (rc != 0) return rc;
+    if (n == 0 || batch == 0) return 0;
+    if (src == nullptr) return -4;
+    if (dst == nullptr) return -5;
+    const int64_t inter = batch_interleaved_elems(n, batch, chunk);
+    const int64_t canon = batch * (int64_t)n * n;
+    const int64_t src_n = dir == 0 ? canon : inter, dst_n = dir == 0 ? inter : canon;
+    const uintptr_t s0 = (uintptr_t)src, s1 = s0 + (uintptr_t)src_n * 4;
+    const uintptr_t d0 = (uintptr_t)dst, d1 = d0 + (uintptr_t)dst_n * 4;
+    if (s0 < d1 && d0 < s1) return -5;
+    const cudaError_t e = launch_convert(dir, n, batch, chunk > 0 ? chunk : batch, src, dst,
+                                         (cudaStream_t)stream);
+    return e == cudaSuccess ? 0 : (int)e;
+}
+
+extern "C" int batch_canonical_to_interleaved(int n, int64_t batch, int chunk, const float *src,
+                                              float *dst, bspotrf_stream_t stream) {
+    return convert_common(0, n, batch, chunk, src, dst, stream);
+}
+
+extern "C" int batch_interleaved_to_canonical(int n, int64_t batch, int chunk, const float *src,
+                                              float *dst, bspotrf_stream_t stream) {
+    return convert_common(1, n, batch, chunk, src, dst, stream);
+}

@@ -1,0 +1,42 @@
+// launch.h -- host-side launcher declarations shared by the C ABI (api.cu)
+// and the per-instance compilation units (gen/inst_*.cu).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace bsp {
+
+struct FactorArgs {
+    float *A;
+    int32_t *info;
+    int32_t *nfailed;    // may be null
+    int64_t batch;
+    int64_t cstride;     // effective chunk C (== batch for simple interleaved)
+    int tpb;             // threads per block (multiple of 32)
+    cudaStream_t stream;
+};
+
+using LaunchFn = cudaError_t (*)(const FactorArgs &);
+
+// Variant REG: lower triangle in registers (csrc/potrf_reg.cuh).
+template <int N, int CT>
+cudaError_t launch_reg(const FactorArgs &a);
+
+// Variant SMEM: left panel of S columns in shared memory, trailing triangle in
+// registers (csrc/potrf_smem.cuh).  TMA: stage with cp.async.bulk (one chunk of
+// CT matrices per block); otherwise per-thread cp.async, per-warp staging.
+template <int N, int CT, int S, bool TMA>
+cudaError_t launch_smem(const FactorArgs &a);
+
+// Variant TILE: the paper's top-looking tile algorithm, NB x NB register
+// tiles streamed from global memory, runtime chunk stride (csrc/potrf_tile.cuh).
+template <int N, int NB>
+cudaError_t launch_tile(const FactorArgs &a);
+
+// Grid size for one-thread-per-matrix kernels.
+inline unsigned grid_for(int64_t batch, int tpb) {
+    return (unsigned)((batch + tpb - 1) / tpb);
+}
+
+}  // namespace bsp

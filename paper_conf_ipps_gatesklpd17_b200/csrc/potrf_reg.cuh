@@ -1,0 +1,76 @@
+// potrf_reg.cuh -- variant REG: one thread per matrix, whole lower triangle in
+// registers, fully unrolled right-looking factorization.
+//
+// This is the paper's fastest kernel shape for n < 20 ("the
+// system is able to preserve data in registers throughout the factorization",
+// PAPER.md:358 "full unrolling pays off up to the size of 20"): Fig. 10's
+// load_lower / store_lower around Fig. 9's spotrf_tile
+// with NB = N.  B200 specifics:
+//  * the unroll is a C++ template on N instead of pyexpander;
+//  * every warp access is one 128-B line (32 lanes x 4 B of 32 consecutive
+//    matrices), issued with streaming cache hints (ld.global.cs / st.global.cs)
+//    because every byte is touched exactly once per launch;
+//  * all N(N+1)/2 loads are issued before the first use (up to 210 independent
+//    LDGs in flight per thread at N = 20), which is what keeps HBM busy;
+//  * column k is stored as soon as it is final, so its registers die early;
+//  * info (LAPACK convention, reading R1) and the fused per-rank failure count
+//    (warp ballot + popc + one atomic per warp) come out of the same kernel.
+#pragma once
+
+#include "common.cuh"
+#include "launch.h"
+
+namespace bsp {
+
+template <int N, int CT>
+__global__ void __launch_bounds__(256)
+potrf_reg_kernel(float *__restrict__ A, int32_t *__restrict__ info,
+                 int32_t *__restrict__ nfailed, int64_t batch, int64_t cs) {
+    constexpr int T = N * (N + 1) / 2;
+    const int64_t gid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const bool active = gid < batch;
+    // Lanes past the end factor a copy of the last matrix (same cache lines,
+    // no extra traffic) and store nothing: no divergence, no pad-lane access.
+    const int64_t g = active ? gid : batch - 1;
+    const Addr<N, CT> ad(A, g, cs);
+
+    float a[T];
+#pragma unroll
+    for (int j = 0; j < N; ++j)
+#pragma unroll
+        for (int i = j; i < N; ++i) a[tri<N>(i, j)] = ld_stream(ad.at(i, j));
+
+    int inf = 0;
+    sfor<0, N>([&](auto k_) {
+        constexpr int k = BSP_CI(k_);
+        const float d = a[tri<N>(k, k)];
+        pivot_check(d, k, inf);
+        const float s = f_sqrt(d);
+        a[tri<N>(k, k)] = s;
+        const float inv = f_rcp(s);
+#pragma unroll
+        for (int m = k + 1; m < N; ++m) a[tri<N>(m, k)] = f_mul(a[tri<N>(m, k)], inv);
+#pragma unroll
+        for (int n = k + 1; n < N; ++n)
+#pragma unroll
+            for (int m = n; m < N; ++m)
+                a[tri<N>(m, n)] = f_upd(a[tri<N>(m, n)], a[tri<N>(m, k)], a[tri<N>(n, k)]);
+        if (active) {
+#pragma unroll
+            for (int m = k; m < N; ++m) st_stream(ad.at(m, k), a[tri<N>(m, k)]);
+        }
+    });
+    if (active) info[gid] = inf;
+    count_failures(active && inf != 0, nfailed);
+}
+
+template <int N, int CT>
+cudaError_t launch_reg(const FactorArgs &a) {
+    const int tpb = a.tpb > 0 ? a.tpb : 128;
+    if (tpb > 256) return cudaErrorInvalidConfiguration;
+    potrf_reg_kernel<N, CT><<<grid_for(a.batch, tpb), tpb, 0, a.stream>>>(
+        a.A, a.info, a.nfailed, a.batch, a.cstride);
+    return cudaGetLastError();
+}
+
+}  // namespace bsp

@@ -23,6 +23,9 @@ Generators (recipes stated in DESIGN.md "Input recipe"):
 * ``als`` ALS-shaped regularised Gram matrix (the workload PAPER.md:22-24
   motivates; parameters are our reading R16 in DESIGN.md).  k_b = 1 + h mod 2n
   "ratings", Y in {-256..255}/256 of shape k_b x n, A = Y^T Y + (k_b/16) I.
+  Y[r, c] = (fmix32(key_b ^ ((r*n + c) * 0x9E3779B1 mod 2^32)) >> 23) - 256
+  with key_b the low 32 bits of h(seed, b, E_Y) and fmix32 MurmurHash3's
+  32-bit finaliser (cheap enough to recompute on the GPU).
   All partial sums are multiples of 2^-16 below 2^8, so A is exact in FP32 for
   any summation order.
 * ``l0``  integer factor (pin P2): L0 strictly-lower in {-3..3}, diag in
@@ -38,7 +41,7 @@ from __future__ import annotations
 import numpy as np
 
 __all__ = [
-    "mix64", "hash3", "generate", "l0_factor", "fail_plan", "expected_fail_count",
+    "mix64", "fmix32", "hash3", "generate", "l0_factor", "fail_plan", "expected_fail_count",
     "UPPER_NAN_BITS", "PAD_BITS", "KINDS",
 ]
 
@@ -69,6 +72,18 @@ def mix64(z):
         z = (z ^ (z >> np.uint64(27))) * _M2
         z = z ^ (z >> np.uint64(31))
     return z
+
+
+def fmix32(x):
+    """MurmurHash3 32-bit finaliser on uint32 arrays (wrapping arithmetic)."""
+    x = np.asarray(x, dtype=np.uint32)
+    with np.errstate(over="ignore"):
+        x = x ^ (x >> np.uint32(16))
+        x = x * np.uint32(0x85EBCA6B)
+        x = x ^ (x >> np.uint32(13))
+        x = x * np.uint32(0xC2B2AE35)
+        x = x ^ (x >> np.uint32(16))
+    return x
 
 
 def hash3(seed, b, e):
@@ -148,14 +163,16 @@ def generate(n, kind, seed, b, upper="mirror", fail_seed=0, fail_period=0):
         low = vals
     elif kind == "als":
         kb = 1 + (hash3(seed, b, E_KB) % np.uint64(2 * n)).astype(np.int64)
+        key = (hash3(seed, b, E_Y) & np.uint64(0xFFFFFFFF)).astype(np.uint32)
         r = np.arange(2 * n)
         c = np.arange(n)
-        e = (E_Y + r[:, None] * n + c[None, :]).astype(np.uint64)       # (2n, n)
+        with np.errstate(over="ignore"):
+            ctr = ((r[:, None] * n + c[None, :]).astype(np.uint32) * np.uint32(0x9E3779B1))
         low = np.empty((B, i.shape[0]), dtype=np.float64)
         step = 2048
         for s in range(0, B, step):
-            hb = hash3(seed, b[s:s + step, None, None], e[None, :, :])
-            Y = (hb >> np.uint64(55)).astype(np.int64) - 256                # (Bs, 2n, n)
+            hb = fmix32(key[s:s + step, None, None] ^ ctr[None, :, :])
+            Y = (hb >> np.uint32(23)).astype(np.int64) - 256                # (Bs, 2n, n)
             Y = np.where(r[None, :, None] < kb[s:s + step, None, None], Y, 0)
             G = np.einsum("kri,krj->kij", Y, Y)                              # exact int64
             A = G[:, i, j].astype(np.float64) / 65536.0

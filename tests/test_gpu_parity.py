@@ -1,0 +1,124 @@
+"""GPU parity: the CUDA path (through the C ABI) against the FP64 oracle.
+
+Bar: info bit-exact (O1); column-normalised factor error
+<= 1e-4 (O2, reading R10); scaled residual <= 10 (O3, R11); strict upper
+triangle and pad lanes bitwise untouched (O4); and -- stronger than the bar --
+bitwise equality with the FP32 Fig. 9 op-order emulator (P8).
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from oracle import layout
+
+import paper_conf_ipps_gatesklpd17_b200 as bsp
+from gpu_helpers import assert_parity, make_batch, run_gpu, torch_mod
+
+pytestmark = pytest.mark.gpu
+
+ALL_N = list(range(1, 33)) + [33, 37, 40, 48, 56, 63, 64]
+
+
+@pytest.mark.parametrize("n", ALL_N)
+def test_parity_chunk32_ragged(n):
+    batch = 3 * 128 + 37          # several blocks / chunks and a ragged tail
+    canon, inter = make_batch(n, batch, 32, kind="dd")
+    out, info, cnt = run_gpu(n, batch, 32, inter)
+    assert_parity(n, batch, 32, canon, inter, out, info, cnt)
+
+
+@pytest.mark.parametrize("n", [1, 2, 5, 8, 13, 16, 20, 21, 24, 27, 32, 40, 64])
+@pytest.mark.parametrize("chunk", [0, 64, 128, 256, 96])
+def test_parity_other_chunks(n, chunk):
+    batch = 301
+    canon, inter = make_batch(n, batch, chunk, kind="als", seed=5)
+    out, info, cnt = run_gpu(n, batch, chunk, inter)
+    assert_parity(n, batch, chunk, canon, inter, out, info, cnt)
+
+
+@pytest.mark.parametrize("n", [1, 3, 8, 16, 21, 25, 32, 33, 64])
+def test_info_exact_with_injected_failures(n):
+    batch = 777
+    canon, inter = make_batch(n, batch, 32, kind="dd", fail_seed=2018, fail_period=7)
+    failed, kk = synth.fail_plan(n, 2018, 7, np.arange(batch, dtype=np.uint64))
+    out, info, cnt = run_gpu(n, batch, 32, inter)
+    assert np.array_equal(info, np.where(failed, kk + 1, 0))
+    assert cnt == int(failed.sum())
+    assert_parity(n, batch, 32, canon, inter, out, info, cnt)
+
+
+@pytest.mark.parametrize("n", [1, 4, 9, 16, 24, 32, 48, 64])
+def test_integer_factor_bit_exact(n):
+    """P2: A = L0 L0^T with integer L0 -> the GPU returns exactly L0."""
+    batch = 200
+    canon, inter = make_batch(n, batch, 32, kind="l0", seed=9)
+    out, info, _ = run_gpu(n, batch, 32, inter)
+    assert (info == 0).all()
+    got = layout.from_interleaved(n, batch, 32, out).reshape(-1, n, n).transpose(0, 2, 1)
+    L0 = synth.l0_factor(n, 9, np.arange(batch, dtype=np.uint64))
+    assert np.array_equal(np.tril(got).astype(np.float64), L0)
+
+
+def _tunings(n, chunk):
+    out = []
+    for tpb in (32, 64, 128, 256):
+        if n <= 24:
+            out.append(dict(variant=bsp.VARIANT_REG, threads_per_block=tpb, param=0, staging=0))
+        for nb in (2, 4, 8):
+            if nb <= n or nb == 2:
+                out.append(dict(variant=bsp.VARIANT_TILE, threads_per_block=tpb, param=nb, staging=0))
+    if 17 <= n <= 32:
+        for s in (n - 16, n - 14, n - 12):
+            if 2 <= s <= n - 2:
+                out.append(dict(variant=bsp.VARIANT_SMEM, threads_per_block=32, param=s, staging=2))
+                out.append(dict(variant=bsp.VARIANT_SMEM, threads_per_block=64, param=s, staging=2))
+                if chunk in (32, 64, 128):
+                    out.append(dict(variant=bsp.VARIANT_SMEM, threads_per_block=0, param=s, staging=1))
+    return out
+
+
+@pytest.mark.parametrize("n", [2, 7, 16, 19, 20, 21, 24, 28, 32, 45, 64])
+@pytest.mark.parametrize("chunk", [32, 64, 0])
+def test_all_variants_bitwise_identical(n, chunk):
+    """P8: every variant / staging / block size gives the same bits."""
+    batch = 2 * 128 + 19
+    canon, inter = make_batch(n, batch, chunk, kind="als", seed=77)
+    ref = None
+    for t in _tunings(n, chunk):
+        out, info, cnt = run_gpu(n, batch, chunk, inter, tune=t)
+        if ref is None:
+            assert_parity(n, batch, chunk, canon, inter, out, info, cnt)
+            ref = (out, info)
+        else:
+            assert np.array_equal(out.view(np.uint32), ref[0].view(np.uint32)), t
+            assert np.array_equal(info, ref[1]), t
+
+
+def test_quick_returns_touch_nothing():
+    torch = torch_mod()
+    A = torch.full((64,), 3.0, device="cuda")
+    info = torch.full((4,), 5, dtype=torch.int32, device="cuda")
+    bsp.batch_spotrf_interleaved(0, 4, 32, A, info)
+    bsp.batch_spotrf_interleaved(4, 0, 32, A, info)
+    torch.cuda.synchronize()
+    assert (A == 3.0).all() and (info == 5).all()
+
+
+def test_single_matrix_and_tiny_batches():
+    for batch in (1, 2, 31, 33):
+        for n in (1, 2, 17, 32):
+            canon, inter = make_batch(n, batch, 32, kind="dd", seed=batch)
+            out, info, cnt = run_gpu(n, batch, 32, inter)
+            assert_parity(n, batch, 32, canon, inter, out, info, cnt)
+
+
+def test_nan_pivot_reported():
+    n, batch = 6, 64
+    canon, _ = make_batch(n, batch, 32, kind="dd", upper="mirror")
+    canon[5, 3 + 3 * n] = np.nan
+    canon[9, 0] = 0.0
+    inter = layout.to_interleaved(n, 32, canon, fill_bits=synth.PAD_BITS)
+    out, info, cnt = run_gpu(n, batch, 32, inter)
+    assert info[5] == 4 and info[9] == 1 and cnt == 2
+    assert (np.delete(info, [5, 9]) == 0).all()
