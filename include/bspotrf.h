@@ -52,9 +52,13 @@ enum {
     BSPOTRF_VARIANT_SMEM = 2, /* left panel of `param` columns staged in shared
                                  memory (TMA bulk or cp.async), trailing
                                  triangle in registers; 2 <= n <= 32           */
-    BSPOTRF_VARIANT_TILE = 3  /* paper's top-looking tile algorithm (Figs. 9-11)
+    BSPOTRF_VARIANT_TILE = 3, /* paper's top-looking tile algorithm (Figs. 9-11)
                                  with param x param register tiles, tiles
                                  streamed from global memory; any n <= 64      */
+    BSPOTRF_VARIANT_PANEL = 4 /* SMEM split with compact code: the panel of
+                                 `param` columns (multiple of 4) factored by a
+                                 rolled 4x4-tile loop in shared memory, rolled
+                                 SYRK, unrolled register tail; 20 <= n <= 32   */
 };
 
 /* Launch tuning (a row of the autotuning table). */
@@ -63,8 +67,11 @@ typedef struct {
     int threads_per_block; /* multiple of 32, 32..1024; 0 = variant default.
                               SMEM variant with TMA staging uses one chunk per
                               block and ignores this.                         */
-    int param;             /* SMEM: panel width s; TILE: tile size nb; REG: 0 */
-    int staging;           /* SMEM only: 0 = auto, 1 = TMA bulk copy
+    int param;             /* SMEM/PANEL: panel width s; TILE: tile size nb;
+                              REG: min resident warps per SM requested from
+                              the compiler (0 = none; 12, 16 for some n;
+                              forces 128 threads per block)                  */
+    int staging;           /* SMEM/PANEL: 0 = auto, 1 = TMA bulk copy
                               (cp.async.bulk, needs chunk in {32,64,128}),
                               2 = per-thread cp.async                         */
 } bspotrf_tuning;

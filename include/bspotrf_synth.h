@@ -41,6 +41,14 @@ int bspotrf_synth_generate(int n, int64_t batch, int chunk, int64_t b0,
 int bspotrf_fill_u32(float *A, int64_t elems, uint32_t value_bits,
                      bspotrf_stream_t stream);
 
+/* Diagnostic "null factorization" (chunk 32 layout only): every thread loads
+ * its matrix's lower triangle exactly as the REG kernel does and stores it
+ * back unchanged, writing info = 0 -- the factorization's memory traffic with
+ * no arithmetic.  n in {4, 8, 16, 20}; tpb multiple of 32 in 32..256.
+ * Errors: -1 n, -2 batch, -3 A/info null, -5 tpb; >0 CUDA error. */
+int bspotrf_probe_copy_lower(int n, int64_t batch, float *A, int32_t *info,
+                             int tpb, bspotrf_stream_t stream);
+
 #ifdef __cplusplus
 }
 #endif

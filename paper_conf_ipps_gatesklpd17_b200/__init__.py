@@ -19,14 +19,14 @@ __all__ = [
     "batch_spotrf_interleaved", "batch_spotrf_interleaved_ex", "bspotrf_get_tuning",
     "batch_canonical_to_interleaved", "batch_interleaved_to_canonical",
     "batch_spotrf_interleaved_host", "batch_spotrf_host_bytes",
-    "bspotrf_synth_generate", "bspotrf_fill_u32", "Tuning",
-    "VARIANT_AUTO", "VARIANT_REG", "VARIANT_SMEM", "VARIANT_TILE",
+    "bspotrf_synth_generate", "bspotrf_fill_u32", "bspotrf_probe_copy_lower", "Tuning",
+    "VARIANT_AUTO", "VARIANT_REG", "VARIANT_SMEM", "VARIANT_TILE", "VARIANT_PANEL",
     "SYNTH_KINDS", "UPPER_MODES", "LIB_PATH",
 ]
 
 LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libbspotrf.so")
 
-VARIANT_AUTO, VARIANT_REG, VARIANT_SMEM, VARIANT_TILE = 0, 1, 2, 3
+VARIANT_AUTO, VARIANT_REG, VARIANT_SMEM, VARIANT_TILE, VARIANT_PANEL = 0, 1, 2, 3, 4
 SYNTH_KINDS = {"dd": 0, "als": 1, "l0": 2}
 UPPER_MODES = {"mirror": 0, "nan": 1, "keep": 2}
 
@@ -35,7 +35,7 @@ EXPORTS = (
     "bspotrf_version", "batch_interleaved_elems", "batch_spotrf_interleaved",
     "batch_spotrf_interleaved_ex", "bspotrf_get_tuning", "batch_canonical_to_interleaved",
     "batch_interleaved_to_canonical", "batch_spotrf_interleaved_host", "batch_spotrf_host_bytes",
-    "bspotrf_synth_generate", "bspotrf_fill_u32",
+    "bspotrf_synth_generate", "bspotrf_fill_u32", "bspotrf_probe_copy_lower",
 )
 
 
@@ -72,6 +72,7 @@ _SIGS = {
     "batch_spotrf_host_bytes": (_i64, [_i32, _i64, _i32]),
     "bspotrf_synth_generate": (_i32, [_i32, _i64, _i32, _i64, _i32, _u64, _i32, _u64, _i64, _vp, _vp]),
     "bspotrf_fill_u32": (_i32, [_vp, _i64, _u32, _vp]),
+    "bspotrf_probe_copy_lower": (_i32, [_i32, _i64, _vp, _vp, _i32, _vp]),
 }
 
 
@@ -210,6 +211,12 @@ def bspotrf_synth_generate(n, batch, chunk, A, kind="dd", seed=2017, b0=0, upper
     return _check("bspotrf_synth_generate", lib().bspotrf_synth_generate(
         n, batch, chunk, b0, SYNTH_KINDS[kind], seed, UPPER_MODES[upper], fail_seed,
         fail_period, _ptr(A), _stream(stream)))
+
+
+def bspotrf_probe_copy_lower(n, batch, A, info, tpb=128, stream=None):
+    """Diagnostic: the REG kernel's memory traffic without arithmetic (chunk 32)."""
+    return _check("bspotrf_probe_copy_lower", lib().bspotrf_probe_copy_lower(
+        n, batch, _ptr(A), _ptr(info), tpb, _stream(stream)))
 
 
 def bspotrf_fill_u32(A, value_bits, elems=None, stream=None):

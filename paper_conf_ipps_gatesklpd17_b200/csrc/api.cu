@@ -18,7 +18,7 @@ cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float
 struct InstEntry {
     int variant;  // BSPOTRF_VARIANT_*
     int n;
-    int param;    // SMEM: S; TILE: NB; REG: 0
+    int param;    // SMEM/PANEL: S; TILE: NB; REG: min warps per SM (0 = none)
     int ct;       // compile-time chunk (0 = runtime stride)
     int tma;      // SMEM staging: 1 = TMA bulk, 0 = cp.async
     LaunchFn fn;
@@ -26,7 +26,7 @@ struct InstEntry {
 
 struct TuneEntry {
     int n;
-    int chunk_class;  // 0: chunk==0 (simple interleaved), 1: chunk>0
+    int chunk;  // exact chunk (0 = simple interleaved), or -1 = any other chunk
     bspotrf_tuning t;
 };
 
@@ -55,12 +55,16 @@ static LaunchFn find(int variant, int n, int param, int ct, int tma) {
 }
 
 static bool default_tuning(int n, int chunk, bspotrf_tuning *t) {
-    for (const auto &e : kTuning) {
-        if (e.n == n && e.chunk_class == (chunk > 0 ? 1 : 0)) {
+    for (const auto &e : kTuning)       // exact (n, chunk) row first
+        if (e.n == n && e.chunk == chunk) {
             *t = e.t;
             return true;
         }
-    }
+    for (const auto &e : kTuning)       // then the row for "any other chunk"
+        if (e.n == n && e.chunk == -1) {
+            *t = e.t;
+            return true;
+        }
     return false;
 }
 
@@ -70,17 +74,18 @@ static LaunchFn resolve(int n, int chunk, const bspotrf_tuning &t, int *tpb_out)
     *tpb_out = t.threads_per_block;
     switch (t.variant) {
     case BSPOTRF_VARIANT_REG:
-        return find(BSPOTRF_VARIANT_REG, n, 0, tmpl_chunk ? chunk : 0, 0);
-    case BSPOTRF_VARIANT_SMEM: {
+        return find(BSPOTRF_VARIANT_REG, n, t.param, tmpl_chunk ? chunk : 0, 0);
+    case BSPOTRF_VARIANT_SMEM:
+    case BSPOTRF_VARIANT_PANEL: {
         int staging = t.staging;
         if (staging == 0) staging = tmpl_chunk ? 1 : 2;
         if (staging == 1) {
             if (!tmpl_chunk) return nullptr;
             *tpb_out = chunk;
-            return find(BSPOTRF_VARIANT_SMEM, n, t.param, chunk, 1);
+            return find(t.variant, n, t.param, chunk, 1);
         }
-        LaunchFn f = find(BSPOTRF_VARIANT_SMEM, n, t.param, chunk == 32 ? 32 : 0, 0);
-        return f ? f : find(BSPOTRF_VARIANT_SMEM, n, t.param, 0, 0);
+        LaunchFn f = find(t.variant, n, t.param, chunk == 32 ? 32 : 0, 0);
+        return f ? f : find(t.variant, n, t.param, 0, 0);
     }
     case BSPOTRF_VARIANT_TILE:
         return find(BSPOTRF_VARIANT_TILE, n, t.param, 0, 0);
@@ -142,6 +147,12 @@ extern "C" int batch_spotrf_interleaved_ex(int n, int64_t batch, int chunk, floa
     }
     int tpb = 0;
     LaunchFn fn = resolve(n, chunk, t, &tpb);
+    if (fn == nullptr && tune == nullptr &&
+        (t.variant == BSPOTRF_VARIANT_SMEM || t.variant == BSPOTRF_VARIANT_PANEL)) {
+        t.staging = 2;                       // table row needs TMA: fall back to cp.async
+        if (t.threads_per_block == 0) t.threads_per_block = 32;
+        fn = resolve(n, chunk, t, &tpb);
+    }
     if (fn == nullptr) return -7;
     FactorArgs a;
     a.A = A;

@@ -19,8 +19,9 @@ struct FactorArgs {
 
 using LaunchFn = cudaError_t (*)(const FactorArgs &);
 
-// Variant REG: lower triangle in registers (csrc/potrf_reg.cuh).
-template <int N, int CT>
+// Variant REG: lower triangle in registers (csrc/potrf_reg.cuh); MINW = the
+// minimum resident warps per SM requested from ptxas (0 = no register cap).
+template <int N, int CT, int MINW>
 cudaError_t launch_reg(const FactorArgs &a);
 
 // Variant SMEM: left panel of S columns in shared memory, trailing triangle in
@@ -28,6 +29,11 @@ cudaError_t launch_reg(const FactorArgs &a);
 // CT matrices per block); otherwise per-thread cp.async, per-warp staging.
 template <int N, int CT, int S, bool TMA>
 cudaError_t launch_smem(const FactorArgs &a);
+
+// Variant PANEL: SMEM split with a rolled tile loop for the panel
+// (csrc/potrf_panel.cuh).
+template <int N, int CT, int S, bool TMA>
+cudaError_t launch_panel(const FactorArgs &a);
 
 // Variant TILE: the paper's top-looking tile algorithm, NB x NB register
 // tiles streamed from global memory, runtime chunk stride (csrc/potrf_tile.cuh).

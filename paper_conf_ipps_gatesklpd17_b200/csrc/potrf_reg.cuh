@@ -22,8 +22,11 @@
 
 namespace bsp {
 
-template <int N, int CT>
-__global__ void __launch_bounds__(256)
+// MINW > 0: ask ptxas for at least MINW resident warps per SM (blocks of 128
+// threads), i.e. cap registers at 65536 / (32 * MINW) -- an occupancy axis of
+// the sweep.  MINW == 0: no cap (up to 255 registers).
+template <int N, int CT, int MINW = 0>
+__global__ void __launch_bounds__(MINW ? 128 : 256, MINW ? MINW / 4 : 1)
 potrf_reg_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                  int32_t *__restrict__ nfailed, int64_t batch, int64_t cs) {
     constexpr int T = N * (N + 1) / 2;
@@ -64,11 +67,11 @@ potrf_reg_kernel(float *__restrict__ A, int32_t *__restrict__ info,
     count_failures(active && inf != 0, nfailed);
 }
 
-template <int N, int CT>
+template <int N, int CT, int MINW>
 cudaError_t launch_reg(const FactorArgs &a) {
-    const int tpb = a.tpb > 0 ? a.tpb : 128;
+    const int tpb = MINW ? 128 : (a.tpb > 0 ? a.tpb : 128);
     if (tpb > 256) return cudaErrorInvalidConfiguration;
-    potrf_reg_kernel<N, CT><<<grid_for(a.batch, tpb), tpb, 0, a.stream>>>(
+    potrf_reg_kernel<N, CT, MINW><<<grid_for(a.batch, tpb), tpb, 0, a.stream>>>(
         a.A, a.info, a.nfailed, a.batch, a.cstride);
     return cudaGetLastError();
 }

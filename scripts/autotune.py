@@ -1,0 +1,156 @@
+#!/usr/bin/env python3
+"""Autotuning sweep on the B200 (§II.D).
+
+Exhaustive over the B200 axes (north star (4)):
+  * chunk size C            -- 32, 64, 128, 256, 512 and 0 (simple interleaved)
+  * variant = unroll depth / staging:
+      REG   full unroll, registers only             (paper: fully unrolled, n_b = n)
+      SMEM  full unroll, left panel of S columns in shared memory, staged by
+            TMA bulk copy (staging 1) or per-thread cp.async (staging 2)
+      TILE  tile ops unrolled, outer loops rolled, NB x NB tiles
+            (paper: partially unrolled top-looking, n_b = NB)
+  * threads per block       -- 32..256
+Each point: regenerate the batch in place (device generator), flush L2, time
+ONE launch with CUDA events; median of --reps.  Every point is also checked
+(failure count 0 on SPD input).  Appends JSON lines (resumable).
+
+    python scripts/autotune.py --n 1-32 --chunks 32,64,128,256,512,0 --out gpurun_out/sweep.jsonl
+"""
+import argparse
+import json
+import os
+import statistics
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+import paper_conf_ipps_gatesklpd17_b200 as bsp  # noqa: E402
+
+REG, SMEM, TILE = bsp.VARIANT_REG, bsp.VARIANT_SMEM, bsp.VARIANT_TILE
+
+
+def parse_range(s):
+    out = []
+    for part in s.split(","):
+        if "-" in part:
+            a, b = part.split("-")
+            out += list(range(int(a), int(b) + 1))
+        else:
+            out.append(int(part))
+    return out
+
+
+PANEL = bsp.VARIANT_PANEL
+
+
+def candidates(n, chunk):
+    c = []
+    if n <= 24:
+        for tpb in (32, 64, 128, 256):
+            c.append(dict(variant=REG, threads_per_block=tpb, param=0, staging=0))
+    if 11 <= n <= 17:
+        c.append(dict(variant=REG, threads_per_block=128, param=12, staging=0))
+    if 11 <= n <= 14:
+        c.append(dict(variant=REG, threads_per_block=128, param=16, staging=0))
+    if 20 <= n <= 32:
+        for s in range(4, n - 7, 4):
+            if n - s > 16:
+                continue
+            if chunk in (32, 64, 128):
+                c.append(dict(variant=PANEL, threads_per_block=0, param=s, staging=1))
+            for tpb in (32, 64):
+                c.append(dict(variant=PANEL, threads_per_block=tpb, param=s, staging=2))
+    if 17 <= n <= 32:
+        for s in (n - 16, n - 14, n - 12):
+            if not (2 <= s <= n - 2):
+                continue
+            if chunk in (32, 64, 128):
+                c.append(dict(variant=SMEM, threads_per_block=0, param=s, staging=1))
+            for tpb in (32, 64, 128):
+                c.append(dict(variant=SMEM, threads_per_block=tpb, param=s, staging=2))
+    for nb in (2, 4, 8):
+        if nb <= n or nb == 2:
+            for tpb in (64, 128, 256):
+                c.append(dict(variant=TILE, threads_per_block=tpb, param=nb, staging=0))
+    return c
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--n", default="1-32")
+    ap.add_argument("--chunks", default="32,64,128,256,512,0")
+    ap.add_argument("--batch", type=int, default=1 << 20)
+    ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--out", default="gpurun_out/sweep.jsonl")
+    ap.add_argument("--kind", default="dd")
+    ap.add_argument("--skip-from", action="append", default=[],
+                    help="JSONL files whose points are already measured")
+    ap.add_argument("--variants", default="1,2,3,4")
+    a = ap.parse_args()
+    os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
+    done = set()
+    for path in [a.out] + a.skip_from:
+        if os.path.exists(path):
+            for line in open(path):
+                r = json.loads(line)
+                done.add((r["n"], r["chunk"], r["variant"], r["threads_per_block"], r["param"], r["staging"]))
+    variants = {int(v) for v in a.variants.split(",")}
+    dev = torch.device("cuda", 0)
+    B = a.batch
+    flush = torch.empty(512 << 18, dtype=torch.float32, device=dev)   # 512 MB > L2
+    info = torch.empty(B, dtype=torch.int32, device=dev)
+    cnt = torch.zeros(1, dtype=torch.int32, device=dev)
+    f = open(a.out, "a")
+    t_start = time.time()
+    for n in parse_range(a.n):
+        for chunk in [int(x) for x in a.chunks.split(",")]:
+            elems = bsp.batch_interleaved_elems(n, B, chunk)
+            A = torch.empty(elems, dtype=torch.float32, device=dev)
+            pristine = torch.empty_like(A)
+            bsp.bspotrf_synth_generate(n, B, chunk, pristine, kind=a.kind, seed=2017)
+            for t in candidates(n, chunk):
+                if t["variant"] not in variants:
+                    continue
+                key = (n, chunk, t["variant"], t["threads_per_block"], t["param"], t["staging"])
+                if key in done:
+                    continue
+                times = []
+                err = None
+                for _ in range(a.reps):
+                    A.copy_(pristine)
+                    flush.fill_(1.0)
+                    cnt.zero_()
+                    e0 = torch.cuda.Event(enable_timing=True)
+                    e1 = torch.cuda.Event(enable_timing=True)
+                    e0.record()
+                    try:
+                        bsp.batch_spotrf_interleaved_ex(n, B, chunk, A, info, nfailed=cnt, tune=t)
+                    except bsp.BspotrfError as ex:
+                        err = ex.code
+                        break
+                    e1.record()
+                    torch.cuda.synchronize()
+                    times.append(e0.elapsed_time(e1))
+                    if int(cnt.item()) != 0:
+                        err = "nonzero failure count on SPD input"
+                        break
+                rec = dict(n=n, chunk=chunk, batch=B, **t)
+                if err is not None:
+                    rec["error"] = err
+                else:
+                    ms = statistics.median(times)
+                    rec.update(ms=round(ms, 5), gbs=round(B * (4 * n * (n + 1) + 4) / ms / 1e6, 1),
+                               gflops=round(B * n ** 3 / 3 / ms / 1e6, 1), reps=times)
+                f.write(json.dumps(rec) + "\n")
+                f.flush()
+            del A, pristine
+            torch.cuda.empty_cache()
+        print(f"n={n} done at {time.time() - t_start:.0f}s", flush=True)
+
+
+if __name__ == "__main__":
+    main()

@@ -60,11 +60,23 @@ def test_integer_factor_bit_exact(n):
     assert np.array_equal(np.tril(got).astype(np.float64), L0)
 
 
+def _panel_s(n):
+    return [s for s in range(4, n - 7, 4) if n - s <= 16] if 20 <= n <= 32 else []
+
+
 def _tunings(n, chunk):
     out = []
-    for tpb in (32, 64, 128, 256):
-        if n <= 24:
+    if n <= 24:
+        for tpb in (32, 64, 128, 256):
             out.append(dict(variant=bsp.VARIANT_REG, threads_per_block=tpb, param=0, staging=0))
+    if 11 <= n <= 17:
+        out.append(dict(variant=bsp.VARIANT_REG, threads_per_block=128, param=12, staging=0))
+    for s in _panel_s(n):
+        out.append(dict(variant=bsp.VARIANT_PANEL, threads_per_block=32, param=s, staging=2))
+        out.append(dict(variant=bsp.VARIANT_PANEL, threads_per_block=64, param=s, staging=2))
+        if chunk in (32, 64, 128):
+            out.append(dict(variant=bsp.VARIANT_PANEL, threads_per_block=0, param=s, staging=1))
+    for tpb in (64, 256):
         for nb in (2, 4, 8):
             if nb <= n or nb == 2:
                 out.append(dict(variant=bsp.VARIANT_TILE, threads_per_block=tpb, param=nb, staging=0))
@@ -78,7 +90,7 @@ def _tunings(n, chunk):
     return out
 
 
-@pytest.mark.parametrize("n", [2, 7, 16, 19, 20, 21, 24, 28, 32, 45, 64])
+@pytest.mark.parametrize("n", [2, 7, 13, 16, 19, 20, 21, 23, 24, 27, 28, 31, 32, 45, 64])
 @pytest.mark.parametrize("chunk", [32, 64, 0])
 def test_all_variants_bitwise_identical(n, chunk):
     """P8: every variant / staging / block size gives the same bits."""
