@@ -55,10 +55,14 @@ enum {
     BSPOTRF_VARIANT_TILE = 3, /* paper's top-looking tile algorithm (Figs. 9-11)
                                  with param x param register tiles, tiles
                                  streamed from global memory; any n <= 64      */
-    BSPOTRF_VARIANT_PANEL = 4 /* SMEM split with compact code: the panel of
+    BSPOTRF_VARIANT_PANEL = 4, /* SMEM split with compact code: the panel of
                                  `param` columns (multiple of 4) factored by a
                                  rolled 4x4-tile loop in shared memory, rolled
                                  SYRK, unrolled register tail; 20 <= n <= 32   */
+    BSPOTRF_VARIANT_PTMEM = 5 /* PANEL with the first panel tile columns held in
+                                 Tensor Memory (tcgen05.ld/st), 128-thread
+                                 CTAs with 256 TMEM columns each (two per SM);
+                                 TMA staging needs chunk 32; 24 <= n <= 32    */
 };
 
 /* Launch tuning (a row of the autotuning table). */

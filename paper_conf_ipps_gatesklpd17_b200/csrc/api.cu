@@ -87,6 +87,13 @@ static LaunchFn resolve(int n, int chunk, const bspotrf_tuning &t, int *tpb_out)
         LaunchFn f = find(t.variant, n, t.param, chunk == 32 ? 32 : 0, 0);
         return f ? f : find(t.variant, n, t.param, 0, 0);
     }
+    case BSPOTRF_VARIANT_PTMEM: {
+        int staging = t.staging == 0 ? (chunk == 32 ? 1 : 2) : t.staging;
+        *tpb_out = 128;
+        if (staging == 1) return chunk == 32 ? find(BSPOTRF_VARIANT_PTMEM, n, t.param, 32, 1) : nullptr;
+        LaunchFn f = find(BSPOTRF_VARIANT_PTMEM, n, t.param, chunk == 32 ? 32 : 0, 0);
+        return f ? f : find(BSPOTRF_VARIANT_PTMEM, n, t.param, 0, 0);
+    }
     case BSPOTRF_VARIANT_TILE:
         return find(BSPOTRF_VARIANT_TILE, n, t.param, 0, 0);
     default:

@@ -35,6 +35,11 @@ cudaError_t launch_smem(const FactorArgs &a);
 template <int N, int CT, int S, bool TMA>
 cudaError_t launch_panel(const FactorArgs &a);
 
+// Variant PTMEM: PANEL with the first panel tile columns in Tensor Memory
+// (csrc/potrf_tmem.cuh); 4-warp CTAs, 256 TMEM columns each.
+template <int N, int CT, int S, bool TMA>
+cudaError_t launch_ptmem(const FactorArgs &a);
+
 // Variant TILE: the paper's top-looking tile algorithm, NB x NB register
 // tiles streamed from global memory, runtime chunk stride (csrc/potrf_tile.cuh).
 template <int N, int NB>

@@ -1,0 +1,365 @@
+// potrf_tmem.cuh -- variant PTMEM: the PANEL split with Tensor Memory (TMEM) as
+// a third on-chip storage tier, for 24 <= n <= 32.
+//
+// At n = 32 one matrix's lower triangle is 528 floats.  With registers and
+// shared memory alone (PANEL variant) a B200 SM holds 4 warps of matrices
+// (50 KB of panel per warp), i.e. ONE warp per scheduler, and ncu shows the
+// kernel issue-latency bound (issue active ~32%, "wait" stalls).  TMEM --
+// 256 KB per SM, 128 lanes x 512 columns of 32-bit, otherwise idle in a
+// kernel without MMAs -- is thread-private per lane when each warp touches
+// only its own 32-lane sub-partition (warp w <-> lanes 32*(w%4)..+31), and is
+// addressed by a runtime column index (unlike registers).  So:
+//   * a CTA is 4 warps (one per TMEM sub-partition) and allocates 256 TMEM
+//     columns; two CTAs -> 8 warps per SM (2 per scheduler);
+//   * the panel's first CS columns (as 4x4 tiles, tile-major, 16 columns per
+//     tile, <= 256 columns) live in TMEM: one tcgen05.ld/st .32x32b.x16 moves
+//     a whole tile of a thread's matrix;
+//   * the remaining panel columns CS..S-1 live in shared memory (TMA bulk
+//     staged, one cp.async.bulk per column run of the warp's 32-matrix chunk);
+//   * the trailing (N-S) triangle lives in registers.
+// Arithmetic and op order are exactly the PANEL variant's (rolled left-looking
+// 4x4 tile loop over the panel, rolled SYRK, unrolled register tail), hence
+// bitwise identical to every other variant (pin P8).
+#pragma once
+
+#include "common.cuh"
+#include "launch.h"
+#include "ptx.cuh"
+
+namespace bsp {
+
+// ---- tcgen05 TMEM primitives (warp-collective, .sync.aligned) --------------
+__device__ __forceinline__ void tmem_alloc(uint32_t *dst_smem, uint32_t ncols) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(dst_smem)),
+                 "r"(ncols)
+                 : "memory");
+}
+__device__ __forceinline__ void tmem_relinquish() {
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_dealloc(uint32_t taddr, uint32_t ncols) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(taddr), "r"(ncols) : "memory");
+}
+__device__ __forceinline__ void tmem_fence_before() {
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_fence_after() {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, float *v) {
+    uint32_t r[16];
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+        : "r"(taddr)
+        : "memory");
+#pragma unroll
+    for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+}
+__device__ __forceinline__ void tmem_ld4(uint32_t taddr, float *v) {
+    uint32_t r[4];
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x4.b32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3])
+                 : "r"(taddr)
+                 : "memory");
+#pragma unroll
+    for (int i = 0; i < 4; ++i) v[i] = __uint_as_float(r[i]);
+}
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const float *v) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
+            taddr),
+        "r"(__float_as_uint(v[0])), "r"(__float_as_uint(v[1])), "r"(__float_as_uint(v[2])),
+        "r"(__float_as_uint(v[3])), "r"(__float_as_uint(v[4])), "r"(__float_as_uint(v[5])),
+        "r"(__float_as_uint(v[6])), "r"(__float_as_uint(v[7])), "r"(__float_as_uint(v[8])),
+        "r"(__float_as_uint(v[9])), "r"(__float_as_uint(v[10])), "r"(__float_as_uint(v[11])),
+        "r"(__float_as_uint(v[12])), "r"(__float_as_uint(v[13])), "r"(__float_as_uint(v[14])),
+        "r"(__float_as_uint(v[15]))
+        : "memory");
+}
+
+// ---- shape ------------------------------------------------------------------
+template <int N, int S>
+struct TmemShape {
+    static constexpr int NB = 4;
+    static constexpr int TR = (N + NB - 1) / NB;   // tile rows
+    static constexpr int TC = S / NB;              // panel tile columns
+    static constexpr int tiles_in(int tc) { return tc * TR - tc * (tc - 1) / 2; }
+    static constexpr int pick_ct() {               // panel tile columns kept in TMEM
+        int c = 0;
+        while (c < TC && tiles_in(c + 1) * 16 <= 256) ++c;
+        return c;
+    }
+    static constexpr int CTM = pick_ct();
+    static constexpr int CS = CTM * NB;            // panel columns in TMEM
+    static constexpr int NT = N - S;
+    static constexpr int T = NT * (NT + 1) / 2;
+    // shared-memory part: columns CS..S-1, lower-packed
+    static constexpr int PSM = (S * N - S * (S - 1) / 2) - (CS * N - CS * (CS - 1) / 2);
+    static_assert(S % NB == 0, "panel width must be a multiple of 4");
+    static_assert(CTM >= 1, "TMEM must hold at least one tile column");
+};
+
+template <int N, int CT, int S, bool TMA>
+__global__ void __launch_bounds__(128, 2)
+potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
+                   int32_t *__restrict__ nfailed, int64_t batch, int64_t cs) {
+    using SH = TmemShape<N, S>;
+    constexpr int NB = 4, TR = SH::TR, TC = SH::TC, CTM = SH::CTM, CS = SH::CS;
+    constexpr int NT = SH::NT, T = SH::T, PSM = SH::PSM;
+    constexpr int SB0 = CS * N - CS * (CS - 1) / 2;   // pslot of (CS, CS)
+    static_assert(!TMA || CT == 32, "TMA staging here needs chunk 32 (one chunk per warp)");
+
+    extern __shared__ __align__(128) float smem[];
+    __shared__ uint32_t tmem_base_sh;
+    __shared__ __align__(8) uint64_t bars[4];
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t gid = (int64_t)blockIdx.x * 128 + threadIdx.x;
+    const bool active = gid < batch;
+    const int64_t g = active ? gid : batch - 1;
+    const Addr<N, CT> ad(A, g, cs);
+    float *Q = smem + (size_t)warp * (PSM > 0 ? PSM : 1) * 32 + lane;   // lane-private view
+    auto qs = [&](int m, int c) { return (c * N - (c * (c - 1)) / 2 + (m - c)) - SB0; };
+
+    // ---- TMEM: warp 0 allocates 256 columns for the CTA ---------------------
+    if (warp == 0) {
+        tmem_alloc(&tmem_base_sh, 256);
+        tmem_relinquish();
+    }
+    if constexpr (TMA && PSM > 0) {
+        if (lane == 0) {
+            mbar_init(&bars[warp], 1);
+            mbar_fence_init();
+        }
+    }
+    tmem_fence_before();
+    __syncthreads();
+    tmem_fence_after();
+    const uint32_t tbase = tmem_base_sh + ((uint32_t)(32 * (warp & 3)) << 16);
+    auto tidx = [&](int rb, int pb) { return (uint32_t)(pb * TR - pb * (pb - 1) / 2 + (rb - pb)) * 16u; };
+
+    // ---- shared-memory part of the panel: TMA bulk (chunk 32) or cp.async --
+    if constexpr (PSM > 0) {
+        if constexpr (TMA) {
+            if (lane == 0) {
+                int64_t q = ((int64_t)blockIdx.x * 128 + warp * 32) / 32;
+                const int64_t qmax = (batch - 1) / 32;
+                if (q > qmax) q = qmax;          // idle warp past the end: a valid chunk
+                mbar_arrive_expect_tx(&bars[warp], (uint32_t)(PSM * 32 * 4));
+                const float *chunk = A + q * 32 * (N * N);
+#pragma unroll 1
+                for (int c = CS; c < S; ++c)
+                    bulk_g2s(smem + (size_t)warp * PSM * 32 + qs(c, c) * 32, chunk + (c + c * N) * 32,
+                             (uint32_t)((N - c) * 32 * 4), &bars[warp]);
+            }
+        } else {
+#pragma unroll 1
+            for (int c = CS; c < S; ++c)
+#pragma unroll 4
+                for (int m = c; m < N; ++m) cp_async4(Q + qs(m, c) * 32, ad.at(m, c));
+        }
+    }
+
+    // ---- trailing triangle -> registers ------------------------------------
+    float r[T];
+#pragma unroll
+    for (int n = S; n < N; ++n)
+#pragma unroll
+        for (int m = n; m < N; ++m) r[tri<NT>(m - S, n - S)] = ld_stream(ad.at(m, n));
+
+    // ---- TMEM part of the panel: global -> registers -> tcgen05.st ---------
+    sfor<0, CTM>([&](auto pb_) {
+        constexpr int pb = BSP_CI(pb_);
+        sfor<pb, TR>([&](auto rb_) {
+            constexpr int rb = BSP_CI(rb_);
+            float v[16];
+#pragma unroll
+            for (int j = 0; j < NB; ++j)
+#pragma unroll
+                for (int i = 0; i < NB; ++i) {
+                    const int m = rb * NB + i, c = pb * NB + j;
+                    const bool ok = m < N && (rb > pb || i >= j);
+                    v[i + j * NB] = ok ? ld_stream(ad.at(m, c)) : 0.0f;
+                }
+            tmem_st16(tbase + tidx(rb, pb), v);
+        });
+    });
+    tmem_wait_st();
+    if constexpr (PSM > 0) {
+        if constexpr (TMA) mbar_wait(&bars[warp], 0);
+        else cp_async_wait_all();
+    }
+
+    int inf = 0;
+    // tile loader: TMEM (tile columns < CTM) or shared memory (packed)
+    auto load_tile = [&](int rb, int pb, float *t, bool lower_only) {
+        if (pb < CTM) {
+            tmem_ld16(tbase + tidx(rb, pb), t);
+        } else {
+#pragma unroll
+            for (int j = 0; j < NB; ++j)
+#pragma unroll
+                for (int i = 0; i < NB; ++i) {
+                    const int m = rb * NB + i, c = pb * NB + j;
+                    const bool ok = m < N && (!lower_only || i >= j);
+                    t[i + j * NB] = ok ? Q[qs(m, c) * 32] : 0.0f;
+                }
+        }
+    };
+
+    // ---- 1. panel: rolled left-looking over 4x4 tiles -------------------------
+#pragma unroll 1
+    for (int cb = 0; cb < TC; ++cb) {
+#pragma unroll 1
+        for (int rb = cb; rb < TR; ++rb) {
+            const bool diag = rb == cb;
+            float acc[16];
+            load_tile(rb, cb, acc, diag);
+#pragma unroll 1
+            for (int pb = 0; pb < cb; ++pb) {
+                float a[16], b[16];
+                load_tile(rb, pb, a, false);
+                load_tile(cb, pb, b, false);
+                tmem_wait_ld();
+#pragma unroll
+                for (int k = 0; k < NB; ++k)
+#pragma unroll
+                    for (int j = 0; j < NB; ++j)
+#pragma unroll
+                        for (int i = 0; i < NB; ++i)
+                            if (!diag || i >= j)
+                                acc[i + j * NB] = f_upd(acc[i + j * NB], a[i + k * NB], b[j + k * NB]);
+            }
+            tmem_wait_ld();
+            if (diag) {
+#pragma unroll
+                for (int k = 0; k < NB; ++k) {
+                    const float d = acc[k + k * NB];
+                    pivot_check(d, cb * NB + k, inf);
+                    const float s = f_sqrt(d);
+                    acc[k + k * NB] = s;
+                    const float inv = f_rcp(s);
+#pragma unroll
+                    for (int i = k + 1; i < NB; ++i) acc[i + k * NB] = f_mul(acc[i + k * NB], inv);
+#pragma unroll
+                    for (int j = k + 1; j < NB; ++j)
+#pragma unroll
+                        for (int i = j; i < NB; ++i)
+                            acc[i + j * NB] = f_upd(acc[i + j * NB], acc[i + k * NB], acc[j + k * NB]);
+                }
+            } else {
+                float l[16];
+                load_tile(cb, cb, l, true);
+                tmem_wait_ld();
+#pragma unroll
+                for (int k = 0; k < NB; ++k) {
+                    const float inv = f_rcp(l[k + k * NB]);
+#pragma unroll
+                    for (int i = 0; i < NB; ++i) acc[i + k * NB] = f_mul(acc[i + k * NB], inv);
+#pragma unroll
+                    for (int j = k + 1; j < NB; ++j)
+#pragma unroll
+                        for (int i = 0; i < NB; ++i)
+                            acc[i + j * NB] = f_upd(acc[i + j * NB], acc[i + k * NB], l[j + k * NB]);
+                }
+            }
+            // final tile: back to its on-chip home and out to global memory
+            if (cb < CTM) {
+                tmem_st16(tbase + tidx(rb, cb), acc);
+                tmem_wait_st();
+            } else {
+#pragma unroll
+                for (int j = 0; j < NB; ++j)
+#pragma unroll
+                    for (int i = 0; i < NB; ++i) {
+                        const int m = rb * NB + i;
+                        if (m < N && (!diag || i >= j)) Q[qs(m, cb * NB + j) * 32] = acc[i + j * NB];
+                    }
+            }
+            if (active) {
+                float *tb = ad.at(rb * NB, cb * NB);
+#pragma unroll
+                for (int j = 0; j < NB; ++j)
+#pragma unroll
+                    for (int i = 0; i < NB; ++i)
+                        if (rb * NB + i < N && (!diag || i >= j))
+                            st_stream(tb + (int64_t)(i + j * N) * ad.stride(), acc[i + j * NB]);
+            }
+        }
+    }
+
+    // ---- 2. SYRK into the register triangle: rolled over panel columns ------
+    constexpr int RB0 = S / NB;                 // first tile row of the trailing part
+    constexpr int NV = (TR - RB0) * NB;         // >= NT (ragged last tile row)
+#pragma unroll 1
+    for (int k = 0; k < S; ++k) {
+        float v[NV];
+        if (k < CS) {
+            const int pb = k / NB, j = k % NB;
+#pragma unroll
+            for (int rb = RB0; rb < TR; ++rb) tmem_ld4(tbase + tidx(rb, pb) + (uint32_t)(j * NB), v + (rb - RB0) * NB);
+            tmem_wait_ld();
+        } else {
+            const int kb = qs(S, k);
+#pragma unroll
+            for (int m = 0; m < NT; ++m) v[m] = Q[(kb + m) * 32];
+        }
+#pragma unroll
+        for (int n = 0; n < NT; ++n)
+#pragma unroll
+            for (int m = n; m < NT; ++m) r[tri<NT>(m, n)] = f_upd(r[tri<NT>(m, n)], v[m], v[n]);
+    }
+
+    // ---- 3. right-looking on the register triangle (fully unrolled) ----------
+    sfor<0, NT>([&](auto k_) {
+        constexpr int k = BSP_CI(k_);
+        const float d = r[tri<NT>(k, k)];
+        pivot_check(d, k + S, inf);
+        const float s = f_sqrt(d);
+        r[tri<NT>(k, k)] = s;
+        const float inv = f_rcp(s);
+#pragma unroll
+        for (int m = k + 1; m < NT; ++m) r[tri<NT>(m, k)] = f_mul(r[tri<NT>(m, k)], inv);
+#pragma unroll
+        for (int n = k + 1; n < NT; ++n)
+#pragma unroll
+            for (int m = n; m < NT; ++m)
+                r[tri<NT>(m, n)] = f_upd(r[tri<NT>(m, n)], r[tri<NT>(m, k)], r[tri<NT>(n, k)]);
+        if (active) {
+#pragma unroll
+            for (int m = k; m < NT; ++m) st_stream(ad.at(m + S, k + S), r[tri<NT>(m, k)]);
+        }
+    });
+    if (active) info[gid] = inf;
+    count_failures(active && inf != 0, nfailed);
+
+    // ---- release TMEM ---------------------------------------------------------
+    tmem_fence_before();
+    __syncthreads();
+    if (warp == 0) {
+        tmem_fence_after();
+        tmem_dealloc(tmem_base_sh, 256);
+    }
+}
+
+template <int N, int CT, int S, bool TMA>
+cudaError_t launch_ptmem(const FactorArgs &a) {
+    using SH = TmemShape<N, S>;
+    // >= 80 KB of dynamic shared memory keeps at most two CTAs (2 x 256 TMEM
+    // columns) resident per SM, so no CTA ever waits in tcgen05.alloc.
+    size_t sm = (size_t)4 * SH::PSM * 32 * 4;
+    if (sm < 80 * 1024) sm = 80 * 1024;
+    auto kern = potrf_ptmem_kernel<N, CT, S, TMA>;
+    static const cudaError_t once =
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 113 * 1024);
+    if (once != cudaSuccess) return once;
+    kern<<<grid_for(a.batch, 128), 128, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
+    return cudaGetLastError();
+}
+
+}  // namespace bsp

@@ -45,6 +45,7 @@ def parse_range(s):
 
 
 PANEL = bsp.VARIANT_PANEL
+PTMEM = bsp.VARIANT_PTMEM
 
 
 def candidates(n, chunk):
@@ -64,6 +65,13 @@ def candidates(n, chunk):
                 c.append(dict(variant=PANEL, threads_per_block=0, param=s, staging=1))
             for tpb in (32, 64):
                 c.append(dict(variant=PANEL, threads_per_block=tpb, param=s, staging=2))
+    if 24 <= n <= 32:
+        for s in range(4, n - 7, 4):
+            if n - s > 16:
+                continue
+            if chunk == 32:
+                c.append(dict(variant=PTMEM, threads_per_block=128, param=s, staging=1))
+            c.append(dict(variant=PTMEM, threads_per_block=128, param=s, staging=2))
     if 17 <= n <= 32:
         for s in (n - 16, n - 14, n - 12):
             if not (2 <= s <= n - 2):
@@ -89,7 +97,7 @@ def main():
     ap.add_argument("--kind", default="dd")
     ap.add_argument("--skip-from", action="append", default=[],
                     help="JSONL files whose points are already measured")
-    ap.add_argument("--variants", default="1,2,3,4")
+    ap.add_argument("--variants", default="1,2,3,4,5")
     a = ap.parse_args()
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     done = set()

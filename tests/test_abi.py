@@ -85,7 +85,8 @@ def test_tuning_table_covers_every_n(L):
     for n in range(1, 65):
         for chunk in (0, 32, 64):
             t = bsp.bspotrf_get_tuning(n, chunk)
-            assert t.variant in (bsp.VARIANT_REG, bsp.VARIANT_SMEM, bsp.VARIANT_TILE)
+            assert t.variant in (bsp.VARIANT_REG, bsp.VARIANT_SMEM, bsp.VARIANT_TILE,
+                                 bsp.VARIANT_PANEL, bsp.VARIANT_PTMEM)
             assert t.threads_per_block % 32 == 0
     with pytest.raises(bsp.BspotrfError):
         bsp.bspotrf_get_tuning(65, 32)
@@ -98,6 +99,10 @@ def test_explicit_tuning_rejects_unavailable(L):
     assert L.batch_spotrf_interleaved_ex(40, 10, 32, fake, fake, None, ctypes.byref(t), None) == -7
     t = bsp.Tuning(bsp.VARIANT_SMEM, 32, 14, 1)   # TMA staging needs chunk in {32,64,128}
     assert L.batch_spotrf_interleaved_ex(28, 10, 0, fake, fake, None, ctypes.byref(t), None) == -7
+    t = bsp.Tuning(bsp.VARIANT_PTMEM, 128, 16, 1)  # PTMEM TMA staging needs chunk 32
+    assert L.batch_spotrf_interleaved_ex(32, 10, 64, fake, fake, None, ctypes.byref(t), None) == -7
+    t = bsp.Tuning(bsp.VARIANT_PTMEM, 128, 16, 2)  # not instantiated below n = 24
+    assert L.batch_spotrf_interleaved_ex(20, 10, 32, fake, fake, None, ctypes.byref(t), None) == -7
     t = bsp.Tuning(bsp.VARIANT_REG, 48, 0, 0)     # tpb not a multiple of 32
     assert L.batch_spotrf_interleaved_ex(8, 10, 32, fake, fake, None, ctypes.byref(t), None) == -7
 

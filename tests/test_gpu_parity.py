@@ -76,6 +76,11 @@ def _tunings(n, chunk):
         out.append(dict(variant=bsp.VARIANT_PANEL, threads_per_block=64, param=s, staging=2))
         if chunk in (32, 64, 128):
             out.append(dict(variant=bsp.VARIANT_PANEL, threads_per_block=0, param=s, staging=1))
+    if 24 <= n <= 32:
+        for s in _panel_s(n):
+            out.append(dict(variant=bsp.VARIANT_PTMEM, threads_per_block=128, param=s, staging=2))
+            if chunk == 32:
+                out.append(dict(variant=bsp.VARIANT_PTMEM, threads_per_block=128, param=s, staging=1))
     for tpb in (64, 256):
         for nb in (2, 4, 8):
             if nb <= n or nb == 2:
@@ -90,7 +95,7 @@ def _tunings(n, chunk):
     return out
 
 
-@pytest.mark.parametrize("n", [2, 7, 13, 16, 19, 20, 21, 23, 24, 27, 28, 31, 32, 45, 64])
+@pytest.mark.parametrize("n", [2, 7, 13, 16, 19, 20, 21, 23, 24, 25, 27, 28, 29, 30, 31, 32, 45, 64])
 @pytest.mark.parametrize("chunk", [32, 64, 0])
 def test_all_variants_bitwise_identical(n, chunk):
     """P8: every variant / staging / block size gives the same bits."""
