@@ -59,10 +59,13 @@ enum {
                                  `param` columns (multiple of 4) factored by a
                                  rolled 4x4-tile loop in shared memory, rolled
                                  SYRK, unrolled register tail; 20 <= n <= 32   */
-    BSPOTRF_VARIANT_PTMEM = 5 /* PANEL with the first panel tile columns held in
+    BSPOTRF_VARIANT_PTMEM = 5, /* PANEL with the first panel tile columns held in
                                  Tensor Memory (tcgen05.ld/st), 128-thread
                                  CTAs with 256 TMEM columns each (two per SM);
                                  TMA staging needs chunk 32; 24 <= n <= 32    */
+    BSPOTRF_VARIANT_RTMA = 6  /* REG with TMA bulk copies in and out of a
+                                 shared-memory image (chunk 32 only); `param`
+                                 warps per CTA (2 or 4); 4 <= n <= 20         */
 };
 
 /* Launch tuning (a row of the autotuning table). */

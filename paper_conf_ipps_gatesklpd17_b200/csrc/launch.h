@@ -40,6 +40,11 @@ cudaError_t launch_panel(const FactorArgs &a);
 template <int N, int CT, int S, bool TMA>
 cudaError_t launch_ptmem(const FactorArgs &a);
 
+// Variant RTMA: REG with TMA bulk staging in and out (chunk 32 only), W warps
+// per CTA (csrc/potrf_regtma.cuh).
+template <int N, int W>
+cudaError_t launch_regtma(const FactorArgs &a);
+
 // Variant TILE: the paper's top-looking tile algorithm, NB x NB register
 // tiles streamed from global memory, runtime chunk stride (csrc/potrf_tile.cuh).
 template <int N, int NB>

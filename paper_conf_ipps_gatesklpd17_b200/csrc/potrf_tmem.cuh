@@ -356,7 +356,7 @@ cudaError_t launch_ptmem(const FactorArgs &a) {
     if (sm < 80 * 1024) sm = 80 * 1024;
     auto kern = potrf_ptmem_kernel<N, CT, S, TMA>;
     static const cudaError_t once =
-        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 113 * 1024);
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     if (once != cudaSuccess) return once;
     kern<<<grid_for(a.batch, 128), 128, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
     return cudaGetLastError();

@@ -46,6 +46,7 @@ def parse_range(s):
 
 PANEL = bsp.VARIANT_PANEL
 PTMEM = bsp.VARIANT_PTMEM
+RTMA = bsp.VARIANT_RTMA
 
 
 def candidates(n, chunk):
@@ -65,6 +66,9 @@ def candidates(n, chunk):
                 c.append(dict(variant=PANEL, threads_per_block=0, param=s, staging=1))
             for tpb in (32, 64):
                 c.append(dict(variant=PANEL, threads_per_block=tpb, param=s, staging=2))
+    if 4 <= n <= 20 and chunk == 32:
+        for w in (2, 4):
+            c.append(dict(variant=RTMA, threads_per_block=0, param=w, staging=1))
     if 24 <= n <= 32:
         for s in range(4, n - 7, 4):
             if n - s > 16:
@@ -97,7 +101,7 @@ def main():
     ap.add_argument("--kind", default="dd")
     ap.add_argument("--skip-from", action="append", default=[],
                     help="JSONL files whose points are already measured")
-    ap.add_argument("--variants", default="1,2,3,4,5")
+    ap.add_argument("--variants", default="1,2,3,4,5,6")
     a = ap.parse_args()
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     done = set()

@@ -76,6 +76,9 @@ def _tunings(n, chunk):
         out.append(dict(variant=bsp.VARIANT_PANEL, threads_per_block=64, param=s, staging=2))
         if chunk in (32, 64, 128):
             out.append(dict(variant=bsp.VARIANT_PANEL, threads_per_block=0, param=s, staging=1))
+    if 4 <= n <= 20 and chunk == 32:
+        for w in (2, 4):
+            out.append(dict(variant=bsp.VARIANT_RTMA, threads_per_block=0, param=w, staging=1))
     if 24 <= n <= 32:
         for s in _panel_s(n):
             out.append(dict(variant=bsp.VARIANT_PTMEM, threads_per_block=128, param=s, staging=2))
