@@ -140,12 +140,18 @@ int batch_interleaved_to_canonical(int n, int64_t batch, int chunk,
                                    bspotrf_stream_t stream);
 
 /* End-to-end call on HOST buffers (blocking).  hA is the interleaved storage
- * in host memory (pinned memory gives asynchronous, overlapped copies), hinfo
- * host int32[batch], nfailed_out host int32* or NULL (set, not incremented).
- * Only the lower triangle of each matrix crosses PCIe: per column one 2-D copy
- * per slab.  Slabs of `slab` matrices (rounded to whole chunks; 0 = auto) are
- * pipelined over three streams (H2D / factor / D2H) with device workspace from
- * the stream-ordered allocator.  `stream` orders the call after prior work.
+ * in host memory, hinfo host int32[batch], nfailed_out host int32* or NULL
+ * (set, not incremented).  Only the lower triangles cross PCIe.
+ *   slab == 0 and hA, hinfo pinned (page-locked and mapped, e.g.
+ *     cudaHostAlloc / torch pin_memory): ZERO-COPY -- the factorization kernel
+ *     reads and writes the host storage directly over PCIe, one 128-B line per
+ *     warp access, both directions at once;
+ *   otherwise: COPY PIPELINE -- slabs of `slab` matrices (rounded to whole
+ *     chunks; 0 = auto, ~32 MB) flow over three streams (H2D / factor / D2H)
+ *     through device workspace from the stream-ordered allocator; per slab,
+ *     one cudaMemcpy2DAsync per column moves that column's lower runs of every
+ *     chunk (pitch n*n*C); a partial last chunk is copied lane-exactly.
+ * `stream` orders the call after prior work.
  * Errors as batch_spotrf_interleaved, plus -6 slab < 0; positive = CUDA error. */
 int batch_spotrf_interleaved_host(int n, int64_t batch, int chunk, float *hA,
                                   int32_t *hinfo, int32_t *nfailed_out,

@@ -1,6 +1,10 @@
 // host_pipeline.cu -- batch_spotrf_interleaved_host: the end-to-end call on
 // host-resident interleaved storage (include/bspotrf.h).
 //
+// Two paths.  (1) slab == 0 and both host buffers pinned (mapped): zero-copy,
+// the factorization kernel reads and writes host memory directly over PCIe.
+// (2) otherwise: the copy pipeline below.
+//
 // The batch is cut into slabs of whole chunks.  Each slab flows through three
 // streams -- H2D copy, factorization kernel, D2H copy -- with three device
 // buffers in rotation, so PCIe in both directions and the kernel overlap.
@@ -76,6 +80,50 @@ cudaError_t copy_lower(int n, int64_t C, int chunk, int64_t batch, int64_t b0, i
     return e;
 }
 
+// Device view of pinned (page-locked, mapped) host memory, or false.
+bool device_view(void *h, void **d) {
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, h) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    if (at.type != cudaMemoryTypeHost || at.devicePointer == nullptr) return false;
+    *d = at.devicePointer;
+    return true;
+}
+
+// Zero-copy path: the factorization kernel itself reads and writes the pinned
+// host storage over PCIe (every warp access is one 128-B line of 32 matrices,
+// and each thread has its whole triangle's loads in flight, so both PCIe
+// directions stream at once).  TMA-staged variants are swapped for their
+// per-thread-load forms (the bulk engine is not used on host memory).
+int zero_copy(int n, int64_t batch, int chunk, float *dA, int32_t *dinfo, int32_t *nfailed_out,
+              cudaStream_t stream) {
+    bspotrf_tuning t;
+    bspotrf_get_tuning(n, chunk, &t);
+    if (t.variant == BSPOTRF_VARIANT_RTMA) t = bspotrf_tuning{BSPOTRF_VARIANT_REG, 128, 0, 0};
+    if (t.variant == BSPOTRF_VARIANT_SMEM || t.variant == BSPOTRF_VARIANT_PANEL) {
+        t.staging = 2;
+        if (t.threads_per_block == 0) t.threads_per_block = 32;
+    }
+    if (t.variant == BSPOTRF_VARIANT_PTMEM) t.staging = 2;
+    int32_t *dcount = nullptr;
+    cudaError_t e = cudaMallocAsync((void **)&dcount, sizeof(int32_t), stream);
+    if (e != cudaSuccess) return (int)e;
+    int rc = 0;
+    e = cudaMemsetAsync(dcount, 0, sizeof(int32_t), stream);
+    if (e == cudaSuccess) {
+        rc = batch_spotrf_interleaved_ex(n, batch, chunk, dA, dinfo, dcount, &t, (bspotrf_stream_t)stream);
+        if (rc == 0 && nfailed_out)
+            e = cudaMemcpyAsync(nfailed_out, dcount, sizeof(int32_t), cudaMemcpyDeviceToHost, stream);
+    }
+    cudaFreeAsync(dcount, stream);
+    const cudaError_t e2 = cudaStreamSynchronize(stream);
+    if (rc != 0) return rc;
+    if (e != cudaSuccess) return (int)e;
+    return e2 == cudaSuccess ? 0 : (int)e2;
+}
+
 }  // namespace
 
 extern "C" int64_t batch_spotrf_host_bytes(int n, int64_t batch, int chunk) {
@@ -97,10 +145,16 @@ extern "C" int batch_spotrf_interleaved_host(int n, int64_t batch, int chunk, fl
     if (hA == nullptr) return -4;
     if (hinfo == nullptr) return -5;
 
+    void *dA_view = nullptr, *dinfo_view = nullptr;
+    if (slab == 0 && device_view(hA, &dA_view) && device_view(hinfo, &dinfo_view) &&
+        (reinterpret_cast<uintptr_t>(dA_view) & 15u) == 0)
+        return zero_copy(n, batch, chunk, (float *)dA_view, (int32_t *)dinfo_view, nfailed_out,
+                         (cudaStream_t)stream);
+
     const int64_t C = chunk > 0 ? chunk : batch;
     const int64_t lower_bytes = (int64_t)4 * n * (n + 1) / 2;
     int64_t S = slab;
-    if (S == 0) S = std::max<int64_t>(1, (int64_t)(96ll << 20) / lower_bytes);  // ~96 MB per slab
+    if (S == 0) S = std::max<int64_t>(1, (int64_t)(32ll << 20) / lower_bytes);  // ~32 MB per slab
     if (chunk > 0) S = std::max<int64_t>(C, (S / C) * C);
     else S = std::max<int64_t>(32, ((S + 31) / 32) * 32);
     S = std::min<int64_t>(S, chunk > 0 ? ((batch + C - 1) / C) * C : batch);

@@ -232,9 +232,8 @@ cudaError_t launch_panel(const FactorArgs &a) {
     const size_t sm = TMA ? (size_t)SH::PS * CT * 4 + 16 : (size_t)(tpb / 32) * SH::PS * 32 * 4;
     auto kern = potrf_panel_kernel<N, CT, S, TMA>;
     if (sm > 48 * 1024) {
-        static const cudaError_t once = cudaFuncSetAttribute(
-            kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-        if (once != cudaSuccess) return once;
+        const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+        if (e != cudaSuccess) return e;
     }
     kern<<<grid_for(a.batch, tpb), tpb, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
     return cudaGetLastError();

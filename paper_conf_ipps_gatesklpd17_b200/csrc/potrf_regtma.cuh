@@ -116,10 +116,9 @@ cudaError_t launch_regtma(const FactorArgs &a) {
     constexpr int T = N * (N + 1) / 2;
     const size_t sm = (size_t)W * T * 32 * 4;
     auto kern = potrf_regtma_kernel<N, W>;
-    if (sm > 48 * 1024) {
-        static const cudaError_t once =
-            cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-        if (once != cudaSuccess) return once;
+    if (sm > 48 * 1024) {   // opt in to exactly what this launch needs (static smem counts too)
+        const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+        if (e != cudaSuccess) return e;
     }
     kern<<<grid_for(a.batch, W * 32), W * 32, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch);
     return cudaGetLastError();

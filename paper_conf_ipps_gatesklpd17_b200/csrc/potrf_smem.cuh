@@ -174,10 +174,8 @@ cudaError_t launch_smem(const FactorArgs &a) {
     const size_t sm = smem_bytes<N, CT, S, TMA>(tpb);
     auto kern = potrf_smem_kernel<N, CT, S, TMA>;
     if (sm > 48 * 1024) {
-        // once per instance: opt in to > 48 KB of dynamic shared memory
-        static const cudaError_t once = cudaFuncSetAttribute(
-            kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-        if (once != cudaSuccess) return once;
+        const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+        if (e != cudaSuccess) return e;
     }
     kern<<<grid_for(a.batch, tpb), tpb, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
     return cudaGetLastError();

@@ -355,9 +355,8 @@ cudaError_t launch_ptmem(const FactorArgs &a) {
     size_t sm = (size_t)4 * SH::PSM * 32 * 4;
     if (sm < 80 * 1024) sm = 80 * 1024;
     auto kern = potrf_ptmem_kernel<N, CT, S, TMA>;
-    static const cudaError_t once =
-        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-    if (once != cudaSuccess) return once;
+    const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e != cudaSuccess) return e;
     kern<<<grid_for(a.batch, 128), 128, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
     return cudaGetLastError();
 }
