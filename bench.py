@@ -46,6 +46,10 @@ WORKLOADS = {
                desc="BASELINE configs[0]: n=8, batch=16384, chunk 32 (launch/latency-bound)"),
     "c3": dict(n=32, batch=1 << 22, chunk=32, kind="als",
                desc="BASELINE configs[2]: n=32, batch=4M, ALS-shaped regularised Gram, chunk 32"),
+    "c5": dict(n=32, batch=1 << 25, chunk=32, kind="dd", global_batch=True, fail_period=1009,
+               desc="BASELINE configs[4]: n=32, batch=32M (33554432) GLOBAL split over the GPUs "
+                    "(strong scaling), DD SPD with injected failures (1 in 1009), failure-count "
+                    "all-reduce"),
 }
 
 FLAG_NAMES = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
@@ -268,8 +272,14 @@ def run_ours(a, w):
         dist.init_process_group("nccl", device_id=dev)
     bsp.lib()
 
-    n, B, chunk, kind = w["n"], w["batch"], w["chunk"], w["kind"]
-    b0 = rank * B                                # disjoint global indices per rank
+    n, chunk, kind = w["n"], w["chunk"], w["kind"]
+    fail_period = w.get("fail_period", 0)
+    if w.get("global_batch"):                    # strong scaling: split one global batch
+        from paper_conf_ipps_gatesklpd17_b200 import multi_gpu
+        b0, B = multi_gpu.rank_slice(w["batch"], world, rank, chunk)
+    else:                                        # weak scaling: the batch is per GPU
+        B = w["batch"]
+        b0 = rank * B                            # disjoint global indices per rank
     tune = json.loads(a.tune) if a.tune else None
     tsel = bsp.bspotrf_get_tuning(n, chunk).as_dict() if tune is None else tune
     elems = bsp.batch_interleaved_elems(n, B, chunk)
@@ -287,7 +297,8 @@ def run_ours(a, w):
 
     def regen():
         for A, _, cnt in pool:
-            bsp.bspotrf_synth_generate(n, B, chunk, A, kind=kind, seed=2017, b0=b0, stream=stream)
+            bsp.bspotrf_synth_generate(n, B, chunk, A, kind=kind, seed=2017, b0=b0,
+                                       fail_seed=2018, fail_period=fail_period, stream=stream)
             cnt.zero_()
 
     def barrier():
@@ -333,7 +344,7 @@ def run_ours(a, w):
         barrier()
         total_ms += e0.elapsed_time(e1)
         launch_ms += [s.elapsed_time(t) for s, t in ev]
-        fails += sum(int(pool[i][2].item()) for i in range(g))
+        fails += sum(int(pool[i][2].item()) for i in range(g))   # global (all-reduced) counts
         done += g
     t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
     lm = torch.tensor([statistics.mean(launch_ms)], dtype=torch.float64, device=dev)
@@ -341,25 +352,37 @@ def run_ours(a, w):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         dist.all_reduce(lm, op=dist.ReduceOp.MAX)
     total_ms, mean_launch_ms = float(t.item()), float(lm.item())
-    # correctness guard on the timed output (DD/ALS inputs are SPD)
-    bad = sum(int((pool[i][1] != 0).sum().item()) for i in range(min(P, a.steps)))
-    if bad or fails:
-        raise SystemExit(f"bench: {bad} nonzero info / {fails} counted failures on SPD input")
+    # correctness guard on the timed output: SPD input -> no failure; injected
+    # failures -> the global count equals the enumerated plan (pin P10)
+    expect = 0
+    if fail_period:
+        import synth
+        Bg = w["batch"] if w.get("global_batch") else B * world
+        expect = synth.expected_fail_count(n, 2018, fail_period, 0, Bg)
+    last = min(P, a.steps)
+    bad = sum(int((pool[i][1][:B] != 0).sum().item()) for i in range(last))
+    if (not fail_period and bad) or fails != expect * a.steps:
+        raise SystemExit(f"bench: {bad} nonzero info / {fails} counted failures, expected "
+                         f"{expect} per step")
 
     ms_per_step = total_ms / a.steps
-    value = world * B * flops_per_matrix(n) / (ms_per_step * 1e-3) / 1e9
+    Btot = w["batch"] if w.get("global_batch") else world * B
+    value = Btot * flops_per_matrix(n) / (ms_per_step * 1e-3) / 1e9
     alg_bytes = B * bytes_per_matrix(n)
     achieved = alg_bytes / (mean_launch_ms * 1e-3) / 1e9
     peak, peak_src = measured_peak()
-    hbm_gbs = world * alg_bytes / (ms_per_step * 1e-3) / 1e9
+    hbm_gbs = Btot * bytes_per_matrix(n) / (ms_per_step * 1e-3) / 1e9
 
     # ---------------- e2e: the host-buffer C-ABI call, copies inside the timed region
     e2e = None
     del pool
     torch.cuda.empty_cache()
-    if not a.no_e2e and a.e2e_steps > 0:
+    if not a.no_e2e and a.e2e_steps > 0 and elems * 4 > (48 << 30):
+        e2e = {"value": None, "unit": "Gflop/s", "skipped": "host buffer > 48 GiB"}
+    elif not a.no_e2e and a.e2e_steps > 0:
         dA = torch.empty(elems, dtype=torch.float32, device=dev)
-        bsp.bspotrf_synth_generate(n, B, chunk, dA, kind=kind, seed=2017, b0=b0, stream=stream)
+        bsp.bspotrf_synth_generate(n, B, chunk, dA, kind=kind, seed=2017, b0=b0,
+                                   fail_seed=2018, fail_period=fail_period, stream=stream)
         pristine = dA.cpu()
         del dA
         hA = torch.empty(elems, dtype=torch.float32).pin_memory()
@@ -389,7 +412,7 @@ def run_ours(a, w):
         t_zero = e2e_run(0)                         # default: zero-copy on pinned buffers
         slab = max(chunk or 32, ((32 << 20) // (2 * n * (n + 1))) // (chunk or 32) * (chunk or 32))
         t_pipe = e2e_run(slab)                      # the copy pipeline, for comparison
-        gfl = lambda t: round(world * B * flops_per_matrix(n) / t / 1e9, 3)
+        gfl = lambda t: round(Btot * flops_per_matrix(n) / t / 1e9, 3)
         e2e = {"value": gfl(t_zero), "unit": "Gflop/s", "h2d_bytes_per_step": hb,
                "d2h_bytes_per_step": hb + 4 * B + 4, "ms_per_step": round(t_zero * 1e3, 3),
                "path": "batch_spotrf_interleaved_host(slab=0) on pinned host interleaved storage: "
@@ -406,7 +429,8 @@ def run_ours(a, w):
     line = {
         "metric": METRIC, "value": round(value, 3), "unit": "Gflop/s", "n_gpus": world,
         "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(ms_per_step, 5),
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "higher_is_better": True, "scaling": "strong" if w.get("global_batch") else "weak",
+        "vs_baseline": None, "dtype": "f32",
         "data": "synthetic (seeded counter-hash generator on device)",
         "config": dict(config_of(w, a), tuning=tsel),
         "hbm_gbs": round(hbm_gbs, 2),
