@@ -50,35 +50,25 @@ __device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, float *v) {
-    uint32_t r[16];
     asm volatile(
         "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+        : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]), "=f"(v[6]), "=f"(v[7]),
+          "=f"(v[8]), "=f"(v[9]), "=f"(v[10]), "=f"(v[11]), "=f"(v[12]), "=f"(v[13]), "=f"(v[14]), "=f"(v[15])
         : "r"(taddr)
         : "memory");
-#pragma unroll
-    for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
 }
 __device__ __forceinline__ void tmem_ld4(uint32_t taddr, float *v) {
-    uint32_t r[4];
     asm volatile("tcgen05.ld.sync.aligned.32x32b.x4.b32 {%0,%1,%2,%3}, [%4];"
-                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3])
+                 : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3])
                  : "r"(taddr)
                  : "memory");
-#pragma unroll
-    for (int i = 0; i < 4; ++i) v[i] = __uint_as_float(r[i]);
 }
 __device__ __forceinline__ void tmem_st16(uint32_t taddr, const float *v) {
     asm volatile(
         "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
             taddr),
-        "r"(__float_as_uint(v[0])), "r"(__float_as_uint(v[1])), "r"(__float_as_uint(v[2])),
-        "r"(__float_as_uint(v[3])), "r"(__float_as_uint(v[4])), "r"(__float_as_uint(v[5])),
-        "r"(__float_as_uint(v[6])), "r"(__float_as_uint(v[7])), "r"(__float_as_uint(v[8])),
-        "r"(__float_as_uint(v[9])), "r"(__float_as_uint(v[10])), "r"(__float_as_uint(v[11])),
-        "r"(__float_as_uint(v[12])), "r"(__float_as_uint(v[13])), "r"(__float_as_uint(v[14])),
-        "r"(__float_as_uint(v[15]))
+        "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7]),
+        "f"(v[8]), "f"(v[9]), "f"(v[10]), "f"(v[11]), "f"(v[12]), "f"(v[13]), "f"(v[14]), "f"(v[15])
         : "memory");
 }
 
@@ -196,123 +186,152 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
     }
 
     int inf = 0;
-    // tile loader: TMEM (tile columns < CTM) or shared memory (packed)
-    auto load_tile = [&](int rb, int pb, float *t, bool lower_only) {
-        if (pb < CTM) {
-            tmem_ld16(tbase + tidx(rb, pb), t);
+    // smem tile loader (packed columns CS..S-1); rows >= N read as 0
+    auto load_tile_smem = [&](int rb, int pb, float *t, bool lower_only) {
+#pragma unroll
+        for (int j = 0; j < NB; ++j)
+#pragma unroll
+            for (int i = 0; i < NB; ++i) {
+                const int m = rb * NB + i, c = pb * NB + j;
+                const bool ok = m < N && (!lower_only || i >= j);
+                t[i + j * NB] = ok ? Q[qs(m, c) * 32] : 0.0f;
+            }
+    };
+    // acc -= a * b^T restricted to the lower part when DIAG
+    auto gemm = [&](float *acc, const float *a, const float *b, auto diag_) {
+        constexpr bool DIAG = decltype(diag_)::value;
+#pragma unroll
+        for (int k = 0; k < NB; ++k)
+#pragma unroll
+            for (int j = 0; j < NB; ++j)
+#pragma unroll
+                for (int i = 0; i < NB; ++i)
+                    if (!DIAG || i >= j) acc[i + j * NB] = f_upd(acc[i + j * NB], a[i + k * NB], b[j + k * NB]);
+    };
+    // store a final tile of panel tile column CB to its on-chip home and to global
+    auto put_tile = [&](int rb, const float *acc, auto cb_, auto diag_) {
+        constexpr int CB = decltype(cb_)::value;
+        constexpr bool DIAG = decltype(diag_)::value;
+        if constexpr (CB < CTM) {
+            tmem_st16(tbase + tidx(rb, CB), acc);
         } else {
 #pragma unroll
             for (int j = 0; j < NB; ++j)
 #pragma unroll
                 for (int i = 0; i < NB; ++i) {
-                    const int m = rb * NB + i, c = pb * NB + j;
-                    const bool ok = m < N && (!lower_only || i >= j);
-                    t[i + j * NB] = ok ? Q[qs(m, c) * 32] : 0.0f;
+                    const int m = rb * NB + i;
+                    if (m < N && (!DIAG || i >= j)) Q[qs(m, CB * NB + j) * 32] = acc[i + j * NB];
                 }
+        }
+        if (active) {
+            float *tb = ad.at(rb * NB, CB * NB);
+#pragma unroll
+            for (int j = 0; j < NB; ++j)
+#pragma unroll
+                for (int i = 0; i < NB; ++i)
+                    if (rb * NB + i < N && (!DIAG || i >= j))
+                        st_stream(tb + (int64_t)(i + j * N) * ad.stride(), acc[i + j * NB]);
         }
     };
 
-    // ---- 1. panel: rolled left-looking over 4x4 tiles -------------------------
-#pragma unroll 1
-    for (int cb = 0; cb < TC; ++cb) {
-#pragma unroll 1
-        for (int rb = cb; rb < TR; ++rb) {
-            const bool diag = rb == cb;
-            float acc[16];
-            load_tile(rb, cb, acc, diag);
-#pragma unroll 1
-            for (int pb = 0; pb < cb; ++pb) {
-                float a[16], b[16];
-                load_tile(rb, pb, a, false);
-                load_tile(cb, pb, b, false);
-                tmem_wait_ld();
-#pragma unroll
-                for (int k = 0; k < NB; ++k)
-#pragma unroll
-                    for (int j = 0; j < NB; ++j)
-#pragma unroll
-                        for (int i = 0; i < NB; ++i)
-                            if (!diag || i >= j)
-                                acc[i + j * NB] = f_upd(acc[i + j * NB], a[i + k * NB], b[j + k * NB]);
-            }
+    // ---- 1. panel: left-looking over 4x4 tiles; tile columns unrolled at
+    //         compile time, tile rows rolled --------------------------------------
+    sfor<0, TC>([&](auto cb_) {
+        constexpr int CB = BSP_CI(cb_);
+        using TRUE_ = std::integral_constant<bool, true>;
+        using FALSE_ = std::integral_constant<bool, false>;
+        // (a) diagonal tile (CB, CB): SYRK from the tiles to its left, then spotrf_tile
+        float dg[16];
+        if constexpr (CB < CTM) tmem_ld16(tbase + tidx(CB, CB), dg);
+        else load_tile_smem(CB, CB, dg, true);
+        sfor<0, CB>([&](auto pb_) {
+            constexpr int PB = BSP_CI(pb_);
+            float a[16];
+            if constexpr (PB < CTM) tmem_ld16(tbase + tidx(CB, PB), a);
+            else load_tile_smem(CB, PB, a, false);
             tmem_wait_ld();
-            if (diag) {
+            gemm(dg, a, a, TRUE_{});
+        });
+        tmem_wait_ld();
 #pragma unroll
-                for (int k = 0; k < NB; ++k) {
-                    const float d = acc[k + k * NB];
-                    pivot_check(d, cb * NB + k, inf);
-                    const float s = f_sqrt(d);
-                    acc[k + k * NB] = s;
-                    const float inv = f_rcp(s);
+        for (int k = 0; k < NB; ++k) {
+            const float d = dg[k + k * NB];
+            pivot_check(d, CB * NB + k, inf);
+            const float s = f_sqrt(d);
+            dg[k + k * NB] = s;
+            const float inv = f_rcp(s);
 #pragma unroll
-                    for (int i = k + 1; i < NB; ++i) acc[i + k * NB] = f_mul(acc[i + k * NB], inv);
+            for (int i = k + 1; i < NB; ++i) dg[i + k * NB] = f_mul(dg[i + k * NB], inv);
 #pragma unroll
-                    for (int j = k + 1; j < NB; ++j)
+            for (int j = k + 1; j < NB; ++j)
 #pragma unroll
-                        for (int i = j; i < NB; ++i)
-                            acc[i + j * NB] = f_upd(acc[i + j * NB], acc[i + k * NB], acc[j + k * NB]);
+                for (int i = j; i < NB; ++i) dg[i + j * NB] = f_upd(dg[i + j * NB], dg[i + k * NB], dg[j + k * NB]);
+        }
+        put_tile(CB, dg, cb_, TRUE_{});
+        float rinv[NB];
+#pragma unroll
+        for (int k = 0; k < NB; ++k) rinv[k] = f_rcp(dg[k + k * NB]);
+        // (b) off-diagonal tiles (rb, CB), rb > CB: GEMM updates, then strsm_tile
+#pragma unroll 1
+        for (int rb = CB + 1; rb < TR; ++rb) {
+            float acc[16];
+            if constexpr (CB < CTM) tmem_ld16(tbase + tidx(rb, CB), acc);
+            else load_tile_smem(rb, CB, acc, false);
+            sfor<0, CB>([&](auto pb_) {
+                constexpr int PB = BSP_CI(pb_);
+                float a[16], b[16];
+                if constexpr (PB < CTM) {
+                    tmem_ld16(tbase + tidx(rb, PB), a);
+                    tmem_ld16(tbase + tidx(CB, PB), b);
+                } else {
+                    load_tile_smem(rb, PB, a, false);
+                    load_tile_smem(CB, PB, b, false);
                 }
-            } else {
-                float l[16];
-                load_tile(cb, cb, l, true);
                 tmem_wait_ld();
+                gemm(acc, a, b, FALSE_{});
+            });
+            tmem_wait_ld();
 #pragma unroll
-                for (int k = 0; k < NB; ++k) {
-                    const float inv = f_rcp(l[k + k * NB]);
+            for (int k = 0; k < NB; ++k) {
 #pragma unroll
-                    for (int i = 0; i < NB; ++i) acc[i + k * NB] = f_mul(acc[i + k * NB], inv);
+                for (int i = 0; i < NB; ++i) acc[i + k * NB] = f_mul(acc[i + k * NB], rinv[k]);
 #pragma unroll
-                    for (int j = k + 1; j < NB; ++j)
-#pragma unroll
-                        for (int i = 0; i < NB; ++i)
-                            acc[i + j * NB] = f_upd(acc[i + j * NB], acc[i + k * NB], l[j + k * NB]);
-                }
-            }
-            // final tile: back to its on-chip home and out to global memory
-            if (cb < CTM) {
-                tmem_st16(tbase + tidx(rb, cb), acc);
-                tmem_wait_st();
-            } else {
-#pragma unroll
-                for (int j = 0; j < NB; ++j)
-#pragma unroll
-                    for (int i = 0; i < NB; ++i) {
-                        const int m = rb * NB + i;
-                        if (m < N && (!diag || i >= j)) Q[qs(m, cb * NB + j) * 32] = acc[i + j * NB];
-                    }
-            }
-            if (active) {
-                float *tb = ad.at(rb * NB, cb * NB);
-#pragma unroll
-                for (int j = 0; j < NB; ++j)
+                for (int j = k + 1; j < NB; ++j)
 #pragma unroll
                     for (int i = 0; i < NB; ++i)
-                        if (rb * NB + i < N && (!diag || i >= j))
-                            st_stream(tb + (int64_t)(i + j * N) * ad.stride(), acc[i + j * NB]);
+                        acc[i + j * NB] = f_upd(acc[i + j * NB], acc[i + k * NB], dg[j + k * NB]);
             }
+            put_tile(rb, acc, cb_, FALSE_{});
         }
-    }
+        if constexpr (CB < CTM) tmem_wait_st();
+    });
 
     // ---- 2. SYRK into the register triangle: rolled over panel columns ------
     constexpr int RB0 = S / NB;                 // first tile row of the trailing part
     constexpr int NV = (TR - RB0) * NB;         // >= NT (ragged last tile row)
-#pragma unroll 1
-    for (int k = 0; k < S; ++k) {
-        float v[NV];
-        if (k < CS) {
-            const int pb = k / NB, j = k % NB;
-#pragma unroll
-            for (int rb = RB0; rb < TR; ++rb) tmem_ld4(tbase + tidx(rb, pb) + (uint32_t)(j * NB), v + (rb - RB0) * NB);
-            tmem_wait_ld();
-        } else {
-            const int kb = qs(S, k);
-#pragma unroll
-            for (int m = 0; m < NT; ++m) v[m] = Q[(kb + m) * 32];
-        }
+    auto syrk = [&](const float *v) {
 #pragma unroll
         for (int n = 0; n < NT; ++n)
 #pragma unroll
             for (int m = n; m < NT; ++m) r[tri<NT>(m, n)] = f_upd(r[tri<NT>(m, n)], v[m], v[n]);
+    };
+#pragma unroll 1
+    for (int k = 0; k < CS; ++k) {              // panel columns held in TMEM
+        float v[NV];
+        const uint32_t col = tbase + (uint32_t)((k / NB) * TR - (k / NB) * ((k / NB) - 1) / 2 - (k / NB)) * 16u +
+                             (uint32_t)((k % NB) * NB);
+#pragma unroll
+        for (int rb = RB0; rb < TR; ++rb) tmem_ld4(col + (uint32_t)rb * 16u, v + (rb - RB0) * NB);
+        tmem_wait_ld();
+        syrk(v);
+    }
+#pragma unroll 1
+    for (int k = CS; k < S; ++k) {              // panel columns held in shared memory
+        float v[NT];
+        const int kb = qs(S, k);
+#pragma unroll
+        for (int m = 0; m < NT; ++m) v[m] = Q[(kb + m) * 32];
+        syrk(v);
     }
 
     // ---- 3. right-looking on the register triangle (fully unrolled) ----------
