@@ -42,29 +42,48 @@ convert_kernel(const float *__restrict__ src, float *__restrict__ dst, int64_t b
     // (idx * m) >> 20 with m = 2^20/ecount + 1 is exact (error < 1/256 < 1/ecount)
     const uint32_t m = (1u << 20) / (uint32_t)ecount + 1u;
 
+    constexpr int PER = CV_R * CV_TE / CV_THREADS;   // 16 elements per thread per phase
+    float v[PER];
     if (DIR == 0) {
-#pragma unroll 4
-        for (int idx = threadIdx.x; idx < n_el; idx += CV_THREADS) {
+        // all 16 loads issued before any shared-memory store: 16 lines in flight per thread
+#pragma unroll
+        for (int k = 0; k < PER; ++k) {
+            const int idx = threadIdx.x + k * CV_THREADS;
             const int r = (int)(((uint32_t)idx * m) >> 20), e = idx - r * ecount;
-            if (r < rcount) tile[r][e] = src[cbase + (r0 + r) * E + e0 + e];
+            v[k] = (idx < n_el && r < rcount) ? src[cbase + (r0 + r) * E + e0 + e] : 0.0f;
+        }
+#pragma unroll
+        for (int k = 0; k < PER; ++k) {
+            const int idx = threadIdx.x + k * CV_THREADS;
+            const int r = (int)(((uint32_t)idx * m) >> 20), e = idx - r * ecount;
+            if (idx < n_el) tile[r][e] = v[k];
         }
         __syncthreads();
-#pragma unroll 4
-        for (int idx = threadIdx.x; idx < n_el; idx += CV_THREADS) {
+#pragma unroll
+        for (int k = 0; k < PER; ++k) {
+            const int idx = threadIdx.x + k * CV_THREADS;
             const int e = idx >> 5, r = idx & 31;
-            if (r < rcount) dst[cbase + (int64_t)(e0 + e) * C + r0 + r] = tile[r][e];
+            if (idx < n_el && r < rcount) dst[cbase + (int64_t)(e0 + e) * C + r0 + r] = tile[r][e];
         }
     } else {
-#pragma unroll 4
-        for (int idx = threadIdx.x; idx < n_el; idx += CV_THREADS) {
+#pragma unroll
+        for (int k = 0; k < PER; ++k) {
+            const int idx = threadIdx.x + k * CV_THREADS;
             const int e = idx >> 5, r = idx & 31;
-            if (r < rcount) tile[r][e] = src[cbase + (int64_t)(e0 + e) * C + r0 + r];
+            v[k] = (idx < n_el && r < rcount) ? src[cbase + (int64_t)(e0 + e) * C + r0 + r] : 0.0f;
+        }
+#pragma unroll
+        for (int k = 0; k < PER; ++k) {
+            const int idx = threadIdx.x + k * CV_THREADS;
+            const int e = idx >> 5, r = idx & 31;
+            if (idx < n_el) tile[r][e] = v[k];
         }
         __syncthreads();
-#pragma unroll 4
-        for (int idx = threadIdx.x; idx < n_el; idx += CV_THREADS) {
+#pragma unroll
+        for (int k = 0; k < PER; ++k) {
+            const int idx = threadIdx.x + k * CV_THREADS;
             const int r = (int)(((uint32_t)idx * m) >> 20), e = idx - r * ecount;
-            if (r < rcount) dst[cbase + (r0 + r) * E + e0 + e] = tile[r][e];
+            if (idx < n_el && r < rcount) dst[cbase + (r0 + r) * E + e0 + e] = tile[r][e];
         }
     }
 }
