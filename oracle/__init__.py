@@ -10,6 +10,7 @@ Contents
 --------
 * ``potrf``            -- FP64 Algorithm 1 over a canonical
                           batch; C in ``cholesky.c`` (see its header).
+* ``potrs``            -- FP64 forward/backward substitution.
 * ``spotrf_fig9_fp32`` -- FP32 op-order emulator of Fig. 9 (debugging aid).
 * ``layout``           -- the interleaved address formula (PAPER.md:130-153,
                           222-231) and plain (de)interleaving by that formula.
@@ -56,6 +57,10 @@ def _load():
             lib.oracle_potrf_batch.argtypes = [
                 ctypes.c_int, ctypes.c_int64, ctypes.c_void_p, ctypes.c_void_p,
                 ctypes.c_void_p, ctypes.c_int]
+            lib.oracle_potrs_batch.restype = ctypes.c_int
+            lib.oracle_potrs_batch.argtypes = [
+                ctypes.c_int, ctypes.c_int, ctypes.c_int64, ctypes.c_void_p, ctypes.c_void_p,
+                ctypes.c_void_p]
             lib.oracle_spotrf_fig9_fp32_batch.restype = ctypes.c_int
             lib.oracle_spotrf_fig9_fp32_batch.argtypes = [
                 ctypes.c_int, ctypes.c_int64, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]
@@ -91,6 +96,21 @@ def potrf(n: int, A, nthreads: int | None = None):
     if rc != 0:
         raise RuntimeError(f"oracle_potrf_batch failed rc={rc}")
     return L, info
+
+
+def potrs(n: int, nrhs: int, L64, B):
+    """FP64 forward + backward substitution with the oracle
+    factor L64 (batch, n*n) float64 and canonical FP32 right-hand sides B
+    (batch, n*nrhs), element (i, r) at i + r*n.  Returns X float64 (batch, n*nrhs)."""
+    L64 = np.ascontiguousarray(np.asarray(L64, dtype=np.float64).reshape(-1, n * n))
+    B = np.ascontiguousarray(np.asarray(B, dtype=np.float32).reshape(-1, n * nrhs))
+    X = np.zeros(B.shape, dtype=np.float64)
+    if B.shape[0] and n and nrhs:
+        rc = _load().oracle_potrs_batch(n, nrhs, B.shape[0], L64.ctypes.data, B.ctypes.data,
+                                        X.ctypes.data)
+        if rc != 0:
+            raise RuntimeError("oracle_potrs_batch failed")
+    return X
 
 
 def spotrf_fig9_fp32(n: int, A):

@@ -101,3 +101,34 @@ def accept(n, A_in, L_test, info_test, L64, info64):
     o3 = np.where(ok_ok, r <= RESID_TOL, True)
     return {"info_ok": o1, "err": e, "resid": np.where(ok_ok, r, 0.0),
             "ok": o1 & o2 & o3}
+
+
+# ---- solve (SPOTRS / SPOSV) --------------------------------
+def solve_residual(n, nrhs, A_in, X, B):
+    """Normwise backward error per matrix, FP64:
+    max_r ||b_r - A x_r||_inf / ((||A||_inf ||x_r||_inf + ||b_r||_inf) * n * eps32),
+    A symmetrised from its FP32 lower triangle.  Acceptance: <= 10."""
+    A = _mats(n, A_in)
+    low = lower_mask(n)[None]
+    Al = np.where(low, A, 0.0)
+    S = Al + np.transpose(np.where(np.tril(np.ones((n, n), bool), -1)[None], Al, 0.0), (0, 2, 1))
+    Xm = np.asarray(X, dtype=np.float64).reshape(-1, nrhs, n).transpose(0, 2, 1)   # [b, i, r]
+    Bm = np.asarray(B, dtype=np.float64).reshape(-1, nrhs, n).transpose(0, 2, 1)
+    R = Bm - S @ Xm
+    an = np.abs(S).sum(axis=2).max(axis=1)[:, None]                                   # ||A||_inf
+    num = np.abs(R).max(axis=1)
+    den = (an * np.abs(Xm).max(axis=1) + np.abs(Bm).max(axis=1)) * n * EPS32
+    with np.errstate(divide="ignore", invalid="ignore"):
+        e = np.where(den > 0, num / den, np.where(num > 0, np.inf, 0.0))
+    return e.max(axis=1) if nrhs else np.zeros(len(an))
+
+
+def solve_forward_error(n, nrhs, X, X64):
+    """max_r ||x_r - x64_r||_inf / ||x64_r||_inf per matrix (diagnostic)."""
+    Xm = np.asarray(X, dtype=np.float64).reshape(-1, nrhs, n)
+    Rm = np.asarray(X64, dtype=np.float64).reshape(-1, nrhs, n)
+    num = np.abs(Xm - Rm).max(axis=2)
+    den = np.abs(Rm).max(axis=2)
+    with np.errstate(divide="ignore", invalid="ignore"):
+        e = np.where(den > 0, num / den, num)
+    return e.max(axis=1)
