@@ -157,6 +157,39 @@ int batch_spotrf_interleaved_host(int n, int64_t batch, int chunk, float *hA,
                                   int32_t *hinfo, int32_t *nfailed_out,
                                   int64_t slab, bspotrf_stream_t stream);
 
+/* ---- Solves -------------------------------------------
+ * "A symmetric positive definite system of linear equations Ax = b can be
+ * solved by computing the Cholesky factorization A = LL^T, and then applying
+ * forward substitution and backward substitution to the vector b using the
+ * factors L and L^T".  Right-hand sides B are n x nrhs per
+ * matrix, column-major, interleaved with the SAME chunk as the matrices:
+ * element (i, r) of matrix b's block at (b/C)*C*n*nrhs + (i + r*n)*C + b%C.
+ * One thread per matrix; FP32 with fma accumulation and reciprocal scaling
+ * (the factorization's conventions). */
+
+/* Floats of the interleaved right-hand-side storage: ceil(batch/C)*C*n*nrhs
+ * (0 for an empty problem, -1 on illegal arguments). */
+int64_t batch_interleaved_rhs_elems(int n, int nrhs, int64_t batch, int chunk);
+
+/* Batched SPOTRS: B := A^-1 B using the factor L written by
+ * batch_spotrf_interleaved (device, read only).  B device, overwritten by X.
+ * Matrices must have factored successfully (info == 0); others produce
+ * undefined X.  Right-hand sides are processed 4/2/1 at a time (L is re-read
+ * per group).  Errors: -1 n, -2 nrhs, -3 batch, -4 chunk, -5 L, -6 B;
+ * -7 no kernel instance (n * group > 128 for every group size). */
+int batch_spotrs_interleaved(int n, int nrhs, int64_t batch, int chunk,
+                             const float *L, float *B, bspotrf_stream_t stream);
+
+/* Batched SPOSV: factor A in place (as batch_spotrf_interleaved_ex) and solve
+ * A X = B.  For n <= 20 and nrhs <= 4 a single fused kernel solves with L still
+ * in registers (L is never re-read); otherwise factor then SPOTRS.  LAPACK
+ * semantics: a matrix with info > 0 keeps its right-hand sides unchanged.
+ * nfailed as in _ex.  Errors: -1 n, -2 nrhs, -3 batch, -4 chunk, -5 A,
+ * -6 B, -7 info. */
+int batch_sposv_interleaved(int n, int nrhs, int64_t batch, int chunk,
+                            float *A, float *B, int32_t *info, int32_t *nfailed,
+                            bspotrf_stream_t stream);
+
 /* Bytes of A the host call moves each way (lower triangles only). */
 int64_t batch_spotrf_host_bytes(int n, int64_t batch, int chunk);
 

@@ -20,6 +20,7 @@ __all__ = [
     "batch_canonical_to_interleaved", "batch_interleaved_to_canonical",
     "batch_spotrf_interleaved_host", "batch_spotrf_host_bytes",
     "bspotrf_synth_generate", "bspotrf_fill_u32", "bspotrf_probe_copy_lower", "Tuning",
+    "batch_interleaved_rhs_elems", "batch_spotrs_interleaved", "batch_sposv_interleaved",
     "VARIANT_AUTO", "VARIANT_REG", "VARIANT_SMEM", "VARIANT_TILE", "VARIANT_PANEL", "VARIANT_PTMEM", "VARIANT_RTMA",
     "SYNTH_KINDS", "UPPER_MODES", "LIB_PATH",
 ]
@@ -37,6 +38,7 @@ EXPORTS = (
     "batch_spotrf_interleaved_ex", "bspotrf_get_tuning", "batch_canonical_to_interleaved",
     "batch_interleaved_to_canonical", "batch_spotrf_interleaved_host", "batch_spotrf_host_bytes",
     "bspotrf_synth_generate", "bspotrf_fill_u32", "bspotrf_probe_copy_lower",
+    "batch_interleaved_rhs_elems", "batch_spotrs_interleaved", "batch_sposv_interleaved",
 )
 
 
@@ -74,6 +76,9 @@ _SIGS = {
     "bspotrf_synth_generate": (_i32, [_i32, _i64, _i32, _i64, _i32, _u64, _i32, _u64, _i64, _vp, _vp]),
     "bspotrf_fill_u32": (_i32, [_vp, _i64, _u32, _vp]),
     "bspotrf_probe_copy_lower": (_i32, [_i32, _i64, _vp, _vp, _i32, _vp]),
+    "batch_interleaved_rhs_elems": (_i64, [_i32, _i32, _i64, _i32]),
+    "batch_spotrs_interleaved": (_i32, [_i32, _i32, _i64, _i32, _vp, _vp, _vp]),
+    "batch_sposv_interleaved": (_i32, [_i32, _i32, _i64, _i32, _vp, _vp, _vp, _vp, _vp]),
 }
 
 
@@ -201,6 +206,33 @@ def batch_spotrf_interleaved_host(n, batch, chunk, hA, hinfo, slab=0, stream=Non
     _check("batch_spotrf_interleaved_host", lib().batch_spotrf_interleaved_host(
         n, batch, chunk, _ptr(hA), _ptr(hinfo), ctypes.addressof(nf), slab, _stream(stream)))
     return nf.value
+
+
+def batch_interleaved_rhs_elems(n: int, nrhs: int, batch: int, chunk: int) -> int:
+    r = lib().batch_interleaved_rhs_elems(n, nrhs, batch, chunk)
+    if r < 0:
+        raise BspotrfError("batch_interleaved_rhs_elems", r)
+    return r
+
+
+def batch_spotrs_interleaved(n, nrhs, batch, chunk, L, B, stream=None):
+    """B := A^-1 B with the factor L from batch_spotrf_interleaved (device)."""
+    if n and nrhs and batch:
+        _need(L, batch_interleaved_elems(n, batch, chunk), "torch.float32", "L")
+        _need(B, batch_interleaved_rhs_elems(n, nrhs, batch, chunk), "torch.float32", "B")
+    return _check("batch_spotrs_interleaved", lib().batch_spotrs_interleaved(
+        n, nrhs, batch, chunk, _ptr(L), _ptr(B), _stream(stream)))
+
+
+def batch_sposv_interleaved(n, nrhs, batch, chunk, A, B, info, nfailed=None, stream=None):
+    """Factor A in place and solve A X = B (fused for n <= 20, nrhs <= 4)."""
+    if n and batch:
+        _need(A, batch_interleaved_elems(n, batch, chunk), "torch.float32", "A")
+        _need(info, batch, "torch.int32", "info")
+        if nrhs:
+            _need(B, batch_interleaved_rhs_elems(n, nrhs, batch, chunk), "torch.float32", "B")
+    return _check("batch_sposv_interleaved", lib().batch_sposv_interleaved(
+        n, nrhs, batch, chunk, _ptr(A), _ptr(B), _ptr(info), _ptr(nfailed), _stream(stream)))
 
 
 def bspotrf_synth_generate(n, batch, chunk, A, kind="dd", seed=2017, b0=0, upper="mirror",

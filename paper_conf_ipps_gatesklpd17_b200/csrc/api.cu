@@ -30,7 +30,16 @@ struct TuneEntry {
     bspotrf_tuning t;
 };
 
-#include "gen/registry.inc"      // kInstances[]
+struct SolveEntry {
+    int kind;  // 0 = potrs (standalone), 1 = sposv (fused)
+    int n;
+    int nr;    // right-hand sides per pass
+    int ct;
+    PotrsFn potrs;
+    SposvFn sposv;
+};
+
+#include "gen/registry.inc"      // kInstances[], kSolveInstances[]
 #include "gen/tuning_table.inc"  // kTuning[]
 
 static inline uint64_t key_of(int variant, int n, int param, int ct, int tma) {
@@ -40,13 +49,26 @@ static inline uint64_t key_of(int variant, int n, int param, int ct, int tma) {
 
 static std::once_flag g_once;
 static std::unordered_map<uint64_t, LaunchFn> *g_inst = nullptr;
+static std::unordered_map<uint64_t, const SolveEntry *> *g_solve = nullptr;
+
+static inline uint64_t solve_key(int kind, int n, int nr, int ct) {
+    return ((uint64_t)kind << 40) | ((uint64_t)n << 24) | ((uint64_t)nr << 12) | (uint64_t)ct;
+}
 
 static void init_tables() {
     std::call_once(g_once, [] {
         auto *m = new std::unordered_map<uint64_t, LaunchFn>();
         for (const auto &e : kInstances) (*m)[key_of(e.variant, e.n, e.param, e.ct, e.tma)] = e.fn;
         g_inst = m;
+        auto *sv = new std::unordered_map<uint64_t, const SolveEntry *>();
+        for (const auto &e : kSolveInstances) (*sv)[solve_key(e.kind, e.n, e.nr, e.ct)] = &e;
+        g_solve = sv;
     });
+}
+
+static const SolveEntry *find_solve(int kind, int n, int nr, int chunk) {
+    auto it = g_solve->find(solve_key(kind, n, nr, chunk == 32 ? 32 : 0));
+    return it == g_solve->end() ? nullptr : it->second;
 }
 
 static LaunchFn find(int variant, int n, int param, int ct, int tma) {
@@ -207,4 +229,73 @@ extern "C" int batch_canonical_to_interleaved(int n, int64_t batch, int chunk, c
 extern "C" int batch_interleaved_to_canonical(int n, int64_t batch, int chunk, const float *src,
                                               float *dst, bspotrf_stream_t stream) {
     return convert_common(1, n, batch, chunk, src, dst, stream);
+}
+
+extern "C" int64_t batch_interleaved_rhs_elems(int n, int nrhs, int64_t batch, int chunk) {
+    if (check_common(n, batch, chunk) != 0 || nrhs < 0) return -1;
+    if (n == 0 || nrhs == 0 || batch == 0) return 0;
+    const int64_t C = chunk > 0 ? chunk : batch;
+    return ((batch + C - 1) / C) * C * (int64_t)n * nrhs;
+}
+
+// Standalone solve in groups of 4 / 2 / 1 right-hand sides (L re-read per group).
+static int potrs_groups(const SolveArgs &a, int n, int chunk) {
+    int rhs0 = 0;
+    while (rhs0 < a.nrhs) {
+        const int rem = a.nrhs - rhs0;
+        const SolveEntry *e = nullptr;
+        int nr = 0;
+        for (int cand : {4, 2, 1}) {
+            if (cand > rem) continue;
+            e = find_solve(0, n, cand, chunk);
+            if (e) {
+                nr = cand;
+                break;
+            }
+        }
+        if (e == nullptr) return -7;
+        const cudaError_t err = e->potrs(a, rhs0);
+        if (err != cudaSuccess) return (int)err;
+        rhs0 += nr;
+    }
+    return 0;
+}
+
+extern "C" int batch_spotrs_interleaved(int n, int nrhs, int64_t batch, int chunk, const float *L,
+                                        float *B, bspotrf_stream_t stream) {
+    if (n < 0 || n > BSPOTRF_MAX_N) return -1;
+    if (nrhs < 0) return -2;
+    if (batch < 0) return -3;
+    if (chunk < 0 || (chunk % 32) != 0) return -4;
+    if (n == 0 || nrhs == 0 || batch == 0) return 0;
+    if (L == nullptr) return -5;
+    if (B == nullptr) return -6;
+    init_tables();
+    SolveArgs a{const_cast<float *>(L), B, nullptr, nullptr, batch, chunk > 0 ? chunk : batch, nrhs,
+                (cudaStream_t)stream};
+    return potrs_groups(a, n, chunk);
+}
+
+extern "C" int batch_sposv_interleaved(int n, int nrhs, int64_t batch, int chunk, float *A, float *B,
+                                       int32_t *info, int32_t *nfailed, bspotrf_stream_t stream) {
+    if (n < 0 || n > BSPOTRF_MAX_N) return -1;
+    if (nrhs < 0) return -2;
+    if (batch < 0) return -3;
+    if (chunk < 0 || (chunk % 32) != 0) return -4;
+    if (n == 0 || batch == 0) return 0;
+    if (A == nullptr || (reinterpret_cast<uintptr_t>(A) & 15u) != 0) return -5;
+    if (B == nullptr && nrhs > 0) return -6;
+    if (info == nullptr) return -7;
+    init_tables();
+    SolveArgs a{A, B, info, nfailed, batch, chunk > 0 ? chunk : batch, nrhs, (cudaStream_t)stream};
+    if (nrhs > 0) {
+        if (const SolveEntry *e = find_solve(1, n, nrhs, chunk)) {   // fused: L never re-read
+            const cudaError_t err = e->sposv(a);
+            return err == cudaSuccess ? 0 : (int)err;
+        }
+    }
+    // unfused: factor (tuning table), then solve the matrices whose factorization succeeded
+    const int rc = batch_spotrf_interleaved_ex(n, batch, chunk, A, info, nfailed, nullptr, stream);
+    if (rc != 0 || nrhs == 0) return rc;
+    return potrs_groups(a, n, chunk);
 }

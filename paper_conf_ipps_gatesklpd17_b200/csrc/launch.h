@@ -50,6 +50,24 @@ cudaError_t launch_regtma(const FactorArgs &a);
 template <int N, int NB>
 cudaError_t launch_tile(const FactorArgs &a);
 
+// Solves (csrc/potrs.cuh).
+struct SolveArgs {
+    float *A;       // factor L (spotrs, read) or matrix A (sposv, factored in place)
+    float *B;       // right-hand sides -> solutions
+    int32_t *info;  // sposv only (potrs: nullable "skip failed matrices" mask)
+    int32_t *nfailed;
+    int64_t batch;
+    int64_t cstride;
+    int nrhs;
+    cudaStream_t stream;
+};
+using PotrsFn = cudaError_t (*)(const SolveArgs &, int rhs0);
+using SposvFn = cudaError_t (*)(const SolveArgs &);
+template <int N, int NR, int CT>
+cudaError_t launch_potrs(const SolveArgs &a, int rhs0);
+template <int N, int NR, int CT>
+cudaError_t launch_sposv(const SolveArgs &a);
+
 // Grid size for one-thread-per-matrix kernels.
 inline unsigned grid_for(int64_t batch, int tpb) {
     return (unsigned)((batch + tpb - 1) / tpb);

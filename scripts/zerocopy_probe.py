@@ -3,9 +3,12 @@
 kernel variant (zero-copy: the kernel's loads/stores cross PCIe), vs the copy
 pipeline.  Prints ms and PCIe GB/s each way."""
 import json
+import os
+import sys
 import time
 
-import torch
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
 
 import paper_conf_ipps_gatesklpd17_b200 as bsp
 

@@ -62,6 +62,7 @@ UPPER_NAN_BITS = 0x7FC0FFEE
 PAD_BITS = 0xFFC0DEAD
 
 KINDS = ("dd", "als", "l0")
+E_RHS = 1 << 23       # right-hand sides: B[i, r] uses E_RHS + i + r*n
 
 
 def mix64(z):
@@ -210,3 +211,15 @@ def generate(n, kind, seed, b, upper="mirror", fail_seed=0, fail_period=0):
         raise ValueError(f"unknown upper mode {upper!r}")
     # canonical column-major: flat index i + j*n  ==  transpose to [k, j, i]
     return np.ascontiguousarray(out.transpose(0, 2, 1)).reshape(B, n * n)
+
+
+def generate_rhs(n, nrhs, seed, b):
+    """Right-hand sides for the solve: canonical (len(b), n*nrhs),
+    element (i, r) at i + r*n, values (u16 - 2^15) / 2^12 in [-8, 8) -- exact in FP32."""
+    b = np.atleast_1d(np.asarray(b, dtype=np.uint64))
+    if n == 0 or nrhs == 0 or b.shape[0] == 0:
+        return np.zeros((b.shape[0], n * nrhs), dtype=np.float32)
+    e = (E_RHS + np.arange(n * nrhs)).astype(np.uint64)
+    h = hash3(seed, b[:, None], e[None, :])
+    v = ((h >> np.uint64(48)).astype(np.int64) - (1 << 15)).astype(np.float64) / 4096.0
+    return v.astype(np.float32)

@@ -82,3 +82,14 @@ def test_als_rank_structure():
         ev = np.linalg.eigvalsh(M[t])
         # Y^T Y has rank <= k_b, so at least n - k_b eigenvalues equal the regulariser
         assert (np.abs(ev - reg) < 1e-9).sum() >= max(0, n - kb[t])
+
+
+def test_rhs_generator_exact_and_partition_invariant():
+    n, nrhs = 7, 3
+    B = synth.generate_rhs(n, nrhs, 5, np.arange(100, dtype=np.uint64))
+    assert B.shape == (100, n * nrhs) and B.dtype == np.float32
+    assert np.array_equal(B.astype(np.float64) * 4096, np.round(B.astype(np.float64) * 4096))
+    assert B.min() >= -8 and B.max() < 8
+    part = np.concatenate([synth.generate_rhs(n, nrhs, 5, np.arange(s, s + 50, dtype=np.uint64))
+                           for s in (0, 50)])
+    assert np.array_equal(B.view(np.uint32), part.view(np.uint32))
