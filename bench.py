@@ -213,8 +213,14 @@ def config_of(w, a):
 
 # --------------------------------------------------------------------- clocks
 class ClockSampler:
+    """NVML SM-clock / clock-event-reason sampler.  The thread runs for the
+    whole timed phase; only samples taken inside a marked window (the timed
+    region, bracketed by mark_start/mark_stop) are reported."""
+
     def __init__(self, index):
         self.samples, self.reasons, self.max_mhz = [], 0, None
+        self._all = []
+        self._win = []
         self._stop = threading.Event()
         self._t = None
         try:
@@ -223,6 +229,8 @@ class ClockSampler:
             self.nv = pynvml
             self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
             self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self._rfn = getattr(pynvml, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+                pynvml.nvmlDeviceGetCurrentClocksThrottleReasons
         except Exception:
             self.nv = None
 
@@ -230,30 +238,42 @@ class ClockSampler:
         nv = self.nv
         while not self._stop.is_set():
             try:
-                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
-                fn = getattr(nv, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
-                    nv.nvmlDeviceGetCurrentClocksThrottleReasons
-                self.reasons |= int(fn(self.h))
+                t = time.perf_counter()
+                self._all.append((t, nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM),
+                                  int(self._rfn(self.h))))
             except Exception:
                 pass
-            time.sleep(0.0005)
+            time.sleep(0.0002)
 
     def start(self):
-        if self.nv is not None:
+        if self.nv is not None and self._t is None:
             self._stop.clear()
             self._t = threading.Thread(target=self._run, daemon=True)
             self._t.start()
+            time.sleep(0.002)
+
+    def mark_start(self):
+        self._win.append([time.perf_counter(), None])
+
+    def mark_stop(self):
+        if self._win:
+            self._win[-1][1] = time.perf_counter()
 
     def stop(self):
         if self._t is not None:
             self._stop.set()
             self._t.join()
             self._t = None
+        for t, mhz, r in self._all:
+            if any(a <= t <= (b if b is not None else t) for a, b in self._win):
+                self.samples.append(mhz)
+                self.reasons |= r
 
     def report(self):
         names = [v for k, v in FLAG_NAMES.items() if self.reasons & k and k != 0x1]
         return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
-                "sm_max_mhz": self.max_mhz, "reasons": names, "samples": len(self.samples)}
+                "sm_max_mhz": self.max_mhz, "reasons": names, "samples": len(self.samples),
+                "source": "NVML, sampled every ~0.2 ms inside the timed region"}
 
 
 # --------------------------------------------------------------------- GPU side
@@ -319,6 +339,7 @@ def run_ours(a, w):
     torch.cuda.synchronize(dev)
 
     clk = ClockSampler(local)
+    clk.start()
     total_ms, launch_ms, done = 0.0, [], 0
     fails = 0
     while done < a.steps:
@@ -330,7 +351,7 @@ def run_ours(a, w):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         barrier()
         torch.cuda.synchronize(dev)
-        clk.start()
+        clk.mark_start()
         e0.record(stream)
         for i in range(g):
             ev[i][0].record(stream)
@@ -340,7 +361,7 @@ def run_ours(a, w):
                 dist.all_reduce(pool[i][2])
         e1.record(stream)
         torch.cuda.synchronize(dev)
-        clk.stop()
+        clk.mark_stop()
         barrier()
         total_ms += e0.elapsed_time(e1)
         launch_ms += [s.elapsed_time(t) for s, t in ev]
@@ -352,6 +373,7 @@ def run_ours(a, w):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         dist.all_reduce(lm, op=dist.ReduceOp.MAX)
     total_ms, mean_launch_ms = float(t.item()), float(lm.item())
+    clk.stop()
     # correctness guard on the timed output: SPD input -> no failure; injected
     # failures -> the global count equals the enumerated plan (pin P10)
     expect = 0

@@ -99,14 +99,27 @@ bool device_view(void *h, void **d) {
 // per-thread-load forms (the bulk engine is not used on host memory).
 int zero_copy(int n, int64_t batch, int chunk, float *dA, int32_t *dinfo, int32_t *nfailed_out,
               cudaStream_t stream) {
+    // Kernel choice for PCIe-resident data (scripts/zerocopy_probe.py on B200,
+    // profiles/r01/zerocopy_probe.json): what matters is bytes in flight over
+    // PCIe, not on-chip reuse.  n <= 20: REG, 128 threads (37 GB/s each way at
+    // n=16); 20 < n <= 32: the PANEL split with TMA bulk staging (40 GB/s at
+    // n=32; cp.async.bulk reads mapped host memory fine) where the chunk allows
+    // it, else the table's choice with per-thread staging.
     bspotrf_tuning t;
     bspotrf_get_tuning(n, chunk, &t);
-    if (t.variant == BSPOTRF_VARIANT_RTMA) t = bspotrf_tuning{BSPOTRF_VARIANT_REG, 128, 0, 0};
-    if (t.variant == BSPOTRF_VARIANT_SMEM || t.variant == BSPOTRF_VARIANT_PANEL) {
-        t.staging = 2;
-        if (t.threads_per_block == 0) t.threads_per_block = 32;
+    if (n <= 20) {
+        t = bspotrf_tuning{BSPOTRF_VARIANT_REG, 128, 0, 0};
+    } else if (n <= 32 && (chunk == 32 || chunk == 64 || chunk == 128)) {
+        t = bspotrf_tuning{BSPOTRF_VARIANT_PANEL, 0, n - 16 >= 4 ? ((n - 16 + 3) / 4) * 4 : 4, 1};
+        if (n - t.param > 16 || t.param > n - 8) t.param = ((n - 12) / 4) * 4;
+    } else {
+        if (t.variant == BSPOTRF_VARIANT_RTMA) t = bspotrf_tuning{BSPOTRF_VARIANT_REG, 128, 0, 0};
+        if (t.variant == BSPOTRF_VARIANT_SMEM || t.variant == BSPOTRF_VARIANT_PANEL) {
+            t.staging = 2;
+            if (t.threads_per_block == 0) t.threads_per_block = 32;
+        }
+        if (t.variant == BSPOTRF_VARIANT_PTMEM) t.staging = 2;
     }
-    if (t.variant == BSPOTRF_VARIANT_PTMEM) t.staging = 2;
     int32_t *dcount = nullptr;
     cudaError_t e = cudaMallocAsync((void **)&dcount, sizeof(int32_t), stream);
     if (e != cudaSuccess) return (int)e;
