@@ -271,9 +271,11 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
         float rinv[NB];
 #pragma unroll
         for (int k = 0; k < NB; ++k) rinv[k] = f_rcp(dg[k + k * NB]);
-        // (b) off-diagonal tiles (rb, CB), rb > CB: GEMM updates, then strsm_tile
-#pragma unroll 1
-        for (int rb = CB + 1; rb < TR; ++rb) {
+        // (b) off-diagonal tiles (rb, CB), rb > CB: GEMM updates, then strsm_tile.
+        //     ROWS = real rows of the tile row (4, or N % 4 for a ragged last one,
+        //     peeled so the padded rows cost no arithmetic)
+        auto offdiag = [&](int rb, auto rows_) {
+            constexpr int ROWS = decltype(rows_)::value;
             float acc[16];
             if constexpr (CB < CTM) tmem_ld16(tbase + tidx(rb, CB), acc);
             else load_tile_smem(rb, CB, acc, false);
@@ -288,21 +290,32 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                     load_tile_smem(CB, PB, b, false);
                 }
                 tmem_wait_ld();
-                gemm(acc, a, b, FALSE_{});
+#pragma unroll
+                for (int k = 0; k < NB; ++k)
+#pragma unroll
+                    for (int j = 0; j < NB; ++j)
+#pragma unroll
+                        for (int i = 0; i < ROWS; ++i)
+                            acc[i + j * NB] = f_upd(acc[i + j * NB], a[i + k * NB], b[j + k * NB]);
             });
             tmem_wait_ld();
 #pragma unroll
             for (int k = 0; k < NB; ++k) {
 #pragma unroll
-                for (int i = 0; i < NB; ++i) acc[i + k * NB] = f_mul(acc[i + k * NB], rinv[k]);
+                for (int i = 0; i < ROWS; ++i) acc[i + k * NB] = f_mul(acc[i + k * NB], rinv[k]);
 #pragma unroll
                 for (int j = k + 1; j < NB; ++j)
 #pragma unroll
-                    for (int i = 0; i < NB; ++i)
+                    for (int i = 0; i < ROWS; ++i)
                         acc[i + j * NB] = f_upd(acc[i + j * NB], acc[i + k * NB], dg[j + k * NB]);
             }
             put_tile(rb, acc, cb_, FALSE_{});
-        }
+        };
+        constexpr int TRF = N / NB;                  // full tile rows
+#pragma unroll 1
+        for (int rb = CB + 1; rb < TRF; ++rb) offdiag(rb, std::integral_constant<int, NB>{});
+        if constexpr (N % NB != 0)
+            if constexpr (TR - 1 > CB) offdiag(TR - 1, std::integral_constant<int, N % NB>{});
         if constexpr (CB < CTM) tmem_wait_st();
     });
 
