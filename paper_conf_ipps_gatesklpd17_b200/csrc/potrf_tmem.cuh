@@ -78,10 +78,14 @@ struct TmemShape {
     static constexpr int NB = 4;
     static constexpr int TR = (N + NB - 1) / NB;   // tile rows
     static constexpr int TC = S / NB;              // panel tile columns
+    // TMEM columns per CTA: 256 (two CTAs = 8 warps per SM) up to n = 32; all
+    // 512 (one CTA = 4 warps per SM) for 33 <= n <= 44, where a matrix no
+    // longer fits twice over in registers + shared memory + half the TMEM.
+    static constexpr int COLS = N > 32 ? 512 : 256;
     static constexpr int tiles_in(int tc) { return tc * TR - tc * (tc - 1) / 2; }
     static constexpr int pick_ct() {               // panel tile columns kept in TMEM
         int c = 0;
-        while (c < TC && tiles_in(c + 1) * 16 <= 256) ++c;
+        while (c < TC && tiles_in(c + 1) * 16 <= COLS) ++c;
         return c;
     }
     static constexpr int CTM = pick_ct();
@@ -95,7 +99,7 @@ struct TmemShape {
 };
 
 template <int N, int CT, int S, bool TMA>
-__global__ void __launch_bounds__(128, 2)
+__global__ void __launch_bounds__(128, TmemShape<N, S>::COLS == 256 ? 2 : 1)
 potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                    int32_t *__restrict__ nfailed, int64_t batch, int64_t cs) {
     using SH = TmemShape<N, S>;
@@ -118,7 +122,7 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
 
     // ---- TMEM: warp 0 allocates 256 columns for the CTA ---------------------
     if (warp == 0) {
-        tmem_alloc(&tmem_base_sh, 256);
+        tmem_alloc(&tmem_base_sh, SH::COLS);
         tmem_relinquish();
     }
     if constexpr (TMA && PSM > 0) {
@@ -375,17 +379,19 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
     __syncthreads();
     if (warp == 0) {
         tmem_fence_after();
-        tmem_dealloc(tmem_base_sh, 256);
+        tmem_dealloc(tmem_base_sh, SH::COLS);
     }
 }
 
 template <int N, int CT, int S, bool TMA>
 cudaError_t launch_ptmem(const FactorArgs &a) {
     using SH = TmemShape<N, S>;
-    // >= 80 KB of dynamic shared memory keeps at most two CTAs (2 x 256 TMEM
-    // columns) resident per SM, so no CTA ever waits in tcgen05.alloc.
+    // Enough dynamic shared memory that at most 512 / COLS CTAs are resident
+    // per SM, so no CTA ever waits in tcgen05.alloc: >= 80 KB for two CTAs of
+    // 256 columns, >= 120 KB for one CTA of 512.
     size_t sm = (size_t)4 * SH::PSM * 32 * 4;
-    if (sm < 80 * 1024) sm = 80 * 1024;
+    const size_t floor_sm = SH::COLS == 256 ? 80 * 1024 : 120 * 1024;
+    if (sm < floor_sm) sm = floor_sm;
     auto kern = potrf_ptmem_kernel<N, CT, S, TMA>;
     const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;

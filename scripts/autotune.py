@@ -69,10 +69,10 @@ def candidates(n, chunk):
     if 4 <= n <= 20 and chunk == 32:
         for w in (2, 4):
             c.append(dict(variant=RTMA, threads_per_block=0, param=w, staging=1))
-    if 24 <= n <= 32:
-        for s in range(4, n - 7, 4):
-            if n - s > 16:
-                continue
+    if 24 <= n <= 44:
+        sys.path.insert(0, os.path.join(ROOT, "scripts"))
+        import gen_instances
+        for s in gen_instances.ptmem_s_values(n):
             if chunk == 32:
                 c.append(dict(variant=PTMEM, threads_per_block=128, param=s, staging=1))
             c.append(dict(variant=PTMEM, threads_per_block=128, param=s, staging=2))

@@ -64,6 +64,13 @@ def _panel_s(n):
     return [s for s in range(4, n - 7, 4) if n - s <= 16] if 20 <= n <= 32 else []
 
 
+def _ptmem_s(n):
+    import sys, os
+    sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(__file__)), "scripts"))
+    import gen_instances
+    return gen_instances.ptmem_s_values(n)
+
+
 def _tunings(n, chunk):
     out = []
     if n <= 24:
@@ -79,8 +86,8 @@ def _tunings(n, chunk):
     if 4 <= n <= 20 and chunk == 32:
         for w in (2, 4):
             out.append(dict(variant=bsp.VARIANT_RTMA, threads_per_block=0, param=w, staging=1))
-    if 24 <= n <= 32:
-        for s in _panel_s(n):
+    if 24 <= n <= 44:
+        for s in _ptmem_s(n):
             out.append(dict(variant=bsp.VARIANT_PTMEM, threads_per_block=128, param=s, staging=2))
             if chunk == 32:
                 out.append(dict(variant=bsp.VARIANT_PTMEM, threads_per_block=128, param=s, staging=1))
@@ -98,7 +105,8 @@ def _tunings(n, chunk):
     return out
 
 
-@pytest.mark.parametrize("n", [2, 7, 13, 16, 19, 20, 21, 23, 24, 25, 27, 28, 29, 30, 31, 32, 45, 64])
+@pytest.mark.parametrize("n", [2, 7, 13, 16, 19, 20, 21, 23, 24, 25, 27, 28, 29, 30, 31, 32, 33, 36, 39,
+                               40, 44, 45, 64])
 @pytest.mark.parametrize("chunk", [32, 64, 0])
 def test_all_variants_bitwise_identical(n, chunk):
     """P8: every variant / staging / block size gives the same bits."""
