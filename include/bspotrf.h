@@ -63,9 +63,13 @@ enum {
                                  Tensor Memory (tcgen05.ld/st), 128-thread
                                  CTAs with 256 TMEM columns each (two per SM);
                                  TMA staging needs chunk 32; 24 <= n <= 32    */
-    BSPOTRF_VARIANT_RTMA = 6  /* REG with TMA bulk copies in and out of a
+    BSPOTRF_VARIANT_RTMA = 6, /* REG with TMA bulk copies in and out of a
                                  shared-memory image (chunk 32 only); `param`
                                  warps per CTA (2 or 4); 4 <= n <= 20         */
+    BSPOTRF_VARIANT_RTMAP = 7 /* persistent RTMA: each warp loops over chunks,
+                                 the next chunk's TMA load overlapping this
+                                 chunk's arithmetic; per-thread stores; grid =
+                                 resident warps; chunk 32; 4 <= n <= 20       */
 };
 
 /* Launch tuning (a row of the autotuning table). */

@@ -117,8 +117,9 @@ static LaunchFn resolve(int n, int chunk, const bspotrf_tuning &t, int *tpb_out)
         return f ? f : find(BSPOTRF_VARIANT_PTMEM, n, t.param, 0, 0);
     }
     case BSPOTRF_VARIANT_RTMA:
+    case BSPOTRF_VARIANT_RTMAP:
         *tpb_out = t.param * 32;
-        return chunk == 32 ? find(BSPOTRF_VARIANT_RTMA, n, t.param, 32, 1) : nullptr;
+        return chunk == 32 ? find(t.variant, n, t.param, 32, 1) : nullptr;
     case BSPOTRF_VARIANT_TILE:
         return find(BSPOTRF_VARIANT_TILE, n, t.param, 0, 0);
     default:

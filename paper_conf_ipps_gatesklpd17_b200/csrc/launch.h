@@ -45,6 +45,11 @@ cudaError_t launch_ptmem(const FactorArgs &a);
 template <int N, int W>
 cudaError_t launch_regtma(const FactorArgs &a);
 
+// Variant RTMAP: persistent RTMA, next chunk's TMA load overlapping this
+// chunk's arithmetic (csrc/potrf_regtma.cuh).
+template <int N, int W>
+cudaError_t launch_rtmap(const FactorArgs &a);
+
 // Variant TILE: the paper's top-looking tile algorithm, NB x NB register
 // tiles streamed from global memory, runtime chunk stride (csrc/potrf_tile.cuh).
 template <int N, int NB>

@@ -125,3 +125,105 @@ cudaError_t launch_regtma(const FactorArgs &a) {
 }
 
 }  // namespace bsp
+
+namespace bsp {
+
+// ---- variant RTMAP: persistent RTMA with the next chunk's TMA load in flight
+// during the current chunk's arithmetic ---------------------------------------
+// Each warp loops over chunks (warp-strided).  Its single [slot][lane] image is
+// free as soon as the chunk has been read into registers, so the bulk copies
+// for the NEXT chunk are issued right then and land while this chunk is
+// factored; results leave through per-thread streaming stores (the image is
+// busy with the prefetch).  The grid is exactly the resident warps, so there
+// is no wave tail.
+template <int N, int W>
+__global__ void __launch_bounds__(W * 32, RtmaOcc<N, W>::minb)
+potrf_rtmap_kernel(float *__restrict__ A, int32_t *__restrict__ info,
+                   int32_t *__restrict__ nfailed, int64_t batch) {
+    constexpr int T = N * (N + 1) / 2;
+    extern __shared__ __align__(128) float smem[];
+    __shared__ __align__(8) uint64_t bars[W];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t nchunks = (batch + 31) / 32;
+    const int64_t wstride = (int64_t)gridDim.x * W;
+    int64_t q = (int64_t)blockIdx.x * W + warp;
+    float *img = smem + (size_t)warp * T * 32;
+    uint64_t *bar = &bars[warp];
+    auto issue = [&](int64_t qq) {
+        if (lane == 0) {
+            mbar_arrive_expect_tx(bar, (uint32_t)(T * 32 * 4));
+            const float *chunk = A + qq * 32 * (N * N);
+#pragma unroll 1
+            for (int j = 0; j < N; ++j)
+                bulk_g2s(img + tri<N>(j, j) * 32, chunk + (j + j * N) * 32, (uint32_t)((N - j) * 128), bar);
+        }
+    };
+    if (lane == 0) {
+        mbar_init(bar, 1);
+        mbar_fence_init();
+    }
+    __syncwarp();
+    if (q < nchunks) issue(q);
+    uint32_t phase = 0;
+    for (; q < nchunks; q += wstride) {
+        mbar_wait(bar, phase);
+        phase ^= 1;
+        float a[T];
+#pragma unroll
+        for (int s = 0; s < T; ++s) a[s] = img[s * 32 + lane];
+        // every lane's shared-memory reads must be done before the async proxy
+        // overwrites the image with the next chunk
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        __syncwarp();
+        if (q + wstride < nchunks) issue(q + wstride);
+        const int64_t gid = q * 32 + lane;
+        const bool active = gid < batch;
+        float *cbase = A + q * 32 * (N * N) + lane;
+        int inf = 0;
+        sfor<0, N>([&](auto k_) {
+            constexpr int k = BSP_CI(k_);
+            const float d = a[tri<N>(k, k)];
+            pivot_check(d, k, inf);
+            const float s = f_sqrt(d);
+            a[tri<N>(k, k)] = s;
+            const float inv = f_rcp(s);
+#pragma unroll
+            for (int m = k + 1; m < N; ++m) a[tri<N>(m, k)] = f_mul(a[tri<N>(m, k)], inv);
+#pragma unroll
+            for (int n = k + 1; n < N; ++n)
+#pragma unroll
+                for (int m = n; m < N; ++m)
+                    a[tri<N>(m, n)] = f_upd(a[tri<N>(m, n)], a[tri<N>(m, k)], a[tri<N>(n, k)]);
+            if (active) {
+#pragma unroll
+                for (int m = k; m < N; ++m) st_stream(cbase + (m + k * N) * 32, a[tri<N>(m, k)]);
+            }
+        });
+        if (active) info[gid] = inf;
+        count_failures(active && inf != 0, nfailed);
+    }
+}
+
+template <int N, int W>
+cudaError_t launch_rtmap(const FactorArgs &a) {
+    constexpr int T = N * (N + 1) / 2;
+    const size_t sm = (size_t)W * T * 32 * 4;
+    auto kern = potrf_rtmap_kernel<N, W>;
+    if (sm > 48 * 1024) {
+        const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+        if (e != cudaSuccess) return e;
+    }
+    int dev = 0, sms = 148, per_sm = 1;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, W * 32, sm);
+    if (per_sm < 1) per_sm = 1;
+    const int64_t nchunks = (a.batch + 31) / 32;
+    int64_t grid = (int64_t)sms * per_sm;
+    const int64_t need = (nchunks + W - 1) / W;
+    if (grid > need) grid = need;
+    kern<<<(unsigned)grid, W * 32, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch);
+    return cudaGetLastError();
+}
+
+}  // namespace bsp

@@ -69,6 +69,7 @@ def candidates(n, chunk):
     if 4 <= n <= 20 and chunk == 32:
         for w in (2, 4):
             c.append(dict(variant=RTMA, threads_per_block=0, param=w, staging=1))
+            c.append(dict(variant=bsp.VARIANT_RTMAP, threads_per_block=0, param=w, staging=1))
     if 24 <= n <= 44:
         sys.path.insert(0, os.path.join(ROOT, "scripts"))
         import gen_instances
@@ -101,7 +102,7 @@ def main():
     ap.add_argument("--kind", default="dd")
     ap.add_argument("--skip-from", action="append", default=[],
                     help="JSONL files whose points are already measured")
-    ap.add_argument("--variants", default="1,2,3,4,5,6")
+    ap.add_argument("--variants", default="1,2,3,4,5,6,7")
     a = ap.parse_args()
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     done = set()

@@ -86,7 +86,8 @@ def test_tuning_table_covers_every_n(L):
         for chunk in (0, 32, 64):
             t = bsp.bspotrf_get_tuning(n, chunk)
             assert t.variant in (bsp.VARIANT_REG, bsp.VARIANT_SMEM, bsp.VARIANT_TILE,
-                                 bsp.VARIANT_PANEL, bsp.VARIANT_PTMEM, bsp.VARIANT_RTMA)
+                                 bsp.VARIANT_PANEL, bsp.VARIANT_PTMEM, bsp.VARIANT_RTMA,
+                                 bsp.VARIANT_RTMAP)
             assert t.threads_per_block % 32 == 0
     with pytest.raises(bsp.BspotrfError):
         bsp.bspotrf_get_tuning(65, 32)

@@ -86,6 +86,7 @@ def _tunings(n, chunk):
     if 4 <= n <= 20 and chunk == 32:
         for w in (2, 4):
             out.append(dict(variant=bsp.VARIANT_RTMA, threads_per_block=0, param=w, staging=1))
+            out.append(dict(variant=bsp.VARIANT_RTMAP, threads_per_block=0, param=w, staging=1))
     if 24 <= n <= 44:
         for s in _ptmem_s(n):
             out.append(dict(variant=bsp.VARIANT_PTMEM, threads_per_block=128, param=s, staging=2))
