@@ -57,13 +57,14 @@ __device__ __forceinline__ void cv_issue_loads(const float *__restrict__ src, fl
     const int rcount = (int)((s.batch - m0) < s.R ? (s.batch - m0) : s.R);
     const int n_el = s.R * ecount;
     // idx / ecount without a division: idx < 2^14, ecount <= 128 -> exact
+    // (64-bit product: idx * mg exceeds 2^32 for ecount = 1)
     const uint32_t mg = (1u << 22) / (uint32_t)ecount + 1u;
 #pragma unroll
     for (int k = 0; k < CV_PER; ++k) {
         const int idx = threadIdx.x + k * CV_THREADS;
         if (idx >= n_el) break;
         if (DIR == 0) {                       // canonical rows: lanes -> consecutive elements
-            const int r = (int)(((uint32_t)idx * mg) >> 22), e = idx - r * ecount;
+            const int r = (int)(((uint64_t)idx * mg) >> 22), e = idx - r * ecount;
             if (r < rcount) cp_async4(buf + r * s.ld + e, src + (m0 + r) * s.E + e0 + e);
         } else {                              // interleaved lines: lanes -> consecutive matrices
             const int r = idx & s.rmask, e = idx >> s.rshift;
@@ -89,7 +90,7 @@ __device__ __forceinline__ void cv_store(float *__restrict__ dst, const float *b
             const int r = idx & s.rmask, e = idx >> s.rshift;
             if (r < rcount) dst[gb[r >> 5] + (int64_t)(e0 + e) * s.C + (r & 31)] = buf[r * s.ld + e];
         } else {
-            const int r = (int)(((uint32_t)idx * mg) >> 22), e = idx - r * ecount;
+            const int r = (int)(((uint64_t)idx * mg) >> 22), e = idx - r * ecount;
             if (r < rcount) dst[(m0 + r) * s.E + e0 + e] = buf[r * s.ld + e];
         }
     }
