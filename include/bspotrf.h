@@ -185,8 +185,10 @@ int batch_spotrs_interleaved(int n, int nrhs, int64_t batch, int chunk,
                              const float *L, float *B, bspotrf_stream_t stream);
 
 /* Batched SPOSV: factor A in place (as batch_spotrf_interleaved_ex) and solve
- * A X = B.  For n <= 20 and nrhs <= 4 a single fused kernel solves with L still
- * in registers (L is never re-read); otherwise factor then SPOTRS.  LAPACK
+ * A X = B.  Fused (one kernel, L never re-read) for n <= 20 and nrhs <= 4 (L in
+ * registers) and for 24 <= n <= 44 with nrhs == 1 (L in registers + shared
+ * memory + Tensor Memory, the PTMEM structure); otherwise factor then
+ * SPOTRS.  X is bitwise identical either way.  LAPACK
  * semantics: a matrix with info > 0 keeps its right-hand sides unchanged.
  * nfailed as in _ex.  Errors: -1 n, -2 nrhs, -3 batch, -4 chunk, -5 A,
  * -6 B, -7 info. */

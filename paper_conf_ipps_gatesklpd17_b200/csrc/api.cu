@@ -31,9 +31,9 @@ struct TuneEntry {
 };
 
 struct SolveEntry {
-    int kind;  // 0 = potrs (standalone), 1 = sposv (fused)
+    int kind;  // 0 = potrs (standalone), 1 = sposv (fused, REG), 2 = sposv (fused, PTMEM)
     int n;
-    int nr;    // right-hand sides per pass
+    int nr;    // right-hand sides per pass (kind 2: 2*S + tma)
     int ct;
     PotrsFn potrs;
     SposvFn sposv;
@@ -293,6 +293,22 @@ extern "C" int batch_sposv_interleaved(int n, int nrhs, int64_t batch, int chunk
         if (const SolveEntry *e = find_solve(1, n, nrhs, chunk)) {   // fused: L never re-read
             const cudaError_t err = e->sposv(a);
             return err == cudaSuccess ? 0 : (int)err;
+        }
+        if (nrhs == 1) {                                  // fused on the PTMEM structure
+            bspotrf_tuning t;
+            bspotrf_get_tuning(n, chunk, &t);
+            const bool tma_ok = chunk == 32;
+            const SolveEntry *e = nullptr;
+            if (t.variant == BSPOTRF_VARIANT_PTMEM)
+                e = find_solve(2, n, 2 * t.param + (tma_ok && t.staging != 2 ? 1 : 0), chunk);
+            for (int s : {16, 20, 24, 28, 12, 8}) {
+                if (e == nullptr && tma_ok) e = find_solve(2, n, 2 * s + 1, chunk);
+                if (e == nullptr) e = find_solve(2, n, 2 * s, chunk);
+            }
+            if (e != nullptr) {
+                const cudaError_t err = e->sposv(a);
+                return err == cudaSuccess ? 0 : (int)err;
+            }
         }
     }
     // unfused: factor (tuning table), then solve the matrices whose factorization succeeded

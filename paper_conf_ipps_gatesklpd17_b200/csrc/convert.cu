@@ -11,13 +11,13 @@
 // C % 32 == 0) gives TE segments of 32 contiguous floats -- one 128-B line
 // each.  Both sides fully coalesced.
 //
-// Persistent CTAs (a few per SM) walk the tiles with a two-stage pipeline:
-// the source tile t+1 streams into shared memory with per-thread cp.async
-// (no register staging, 16 copies in flight per thread) while tile t is
-// written out from the other buffer -- so loads are always in flight, which
-// a load-all / sync / store-all kernel cannot sustain.  The padded shared
-// tile (odd pitch) is conflict-free in both directions.  Pad lanes are never
-// touched.
+// Persistent CTAs (the resident count) walk the tiles with a two-stage
+// pipeline in registers: each thread's 16 loads of tile t+1 are issued before
+// tile t is written out of shared memory, so loads stay in flight during the
+// store phase (a load-all / sync / store-all kernel idles HBM reads half the
+// time; per-thread 4-byte cp.async was measured slower: LSU-issue bound).
+// The padded shared tile (odd pitch) is conflict-free in both directions.
+// Pad lanes are never touched.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -37,98 +37,115 @@ struct CvShape {
     int64_t tiles;
 };
 
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int K>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(K) : "memory"); }
 
 // interleaved offset of lane 0 of the 32-matrix group starting at matrix m
 __device__ __forceinline__ int64_t group_base(int64_t m, int64_t C, int E) {
     return (m / C) * C * (int64_t)E + (m % C);
 }
 
-template <int DIR>
-__device__ __forceinline__ void cv_issue_loads(const float *__restrict__ src, float *buf, const CvShape &s,
-                                               int64_t t, const int64_t *gb) {
+// Tile geometry of tile t.
+struct CvTile {
+    int64_t m0;
+    int e0, ecount, rcount, n_el;
+    uint32_t mg;
+};
+__device__ __forceinline__ CvTile cv_tile(const CvShape &s, int64_t t) {
+    CvTile x;
     const int64_t rt = t / s.elem_tiles;
     const int te = (int)(t - rt * s.elem_tiles);
-    const int64_t m0 = rt * s.R;
-    const int e0 = te * s.TE;
-    const int ecount = (s.E - e0) < s.TE ? (s.E - e0) : s.TE;
-    const int rcount = (int)((s.batch - m0) < s.R ? (s.batch - m0) : s.R);
-    const int n_el = s.R * ecount;
+    x.m0 = rt * s.R;
+    x.e0 = te * s.TE;
+    x.ecount = (s.E - x.e0) < s.TE ? (s.E - x.e0) : s.TE;
+    x.rcount = (int)((s.batch - x.m0) < s.R ? (s.batch - x.m0) : s.R);
+    x.n_el = s.R * x.ecount;
     // idx / ecount without a division: idx < 2^14, ecount <= 128 -> exact
     // (64-bit product: idx * mg exceeds 2^32 for ecount = 1)
-    const uint32_t mg = (1u << 22) / (uint32_t)ecount + 1u;
-#pragma unroll
-    for (int k = 0; k < CV_PER; ++k) {
-        const int idx = threadIdx.x + k * CV_THREADS;
-        if (idx >= n_el) break;
-        if (DIR == 0) {                       // canonical rows: lanes -> consecutive elements
-            const int r = (int)(((uint64_t)idx * mg) >> 22), e = idx - r * ecount;
-            if (r < rcount) cp_async4(buf + r * s.ld + e, src + (m0 + r) * s.E + e0 + e);
-        } else {                              // interleaved lines: lanes -> consecutive matrices
-            const int r = idx & s.rmask, e = idx >> s.rshift;
-            if (r < rcount) cp_async4(buf + r * s.ld + e, src + gb[r >> 5] + (int64_t)(e0 + e) * s.C + (r & 31));
-        }
+    x.mg = (1u << 22) / (uint32_t)x.ecount + 1u;
+    return x;
+}
+
+// source element idx of tile x -> (smem slot, global offset); false if padding
+template <int DIR>
+__device__ __forceinline__ bool cv_src(const CvShape &s, const CvTile &x, const int64_t *gb, int idx, int &slot,
+                                       int64_t &off) {
+    if (idx >= x.n_el) return false;
+    int r, e;
+    if (DIR == 0) {                          // canonical rows: lanes -> consecutive elements
+        r = (int)(((uint64_t)idx * x.mg) >> 22);
+        e = idx - r * x.ecount;
+        off = (x.m0 + r) * s.E + x.e0 + e;
+    } else {                                 // interleaved lines: lanes -> consecutive matrices
+        r = idx & s.rmask;
+        e = idx >> s.rshift;
+        off = gb[r >> 5] + (int64_t)(x.e0 + e) * s.C + (r & 31);
     }
+    slot = r * s.ld + e;
+    return r < x.rcount;
 }
 
 template <int DIR>
-__device__ __forceinline__ void cv_store(float *__restrict__ dst, const float *buf, const CvShape &s, int64_t t,
-                                         const int64_t *gb) {
-    const int64_t rt = t / s.elem_tiles;
-    const int te = (int)(t - rt * s.elem_tiles);
-    const int64_t m0 = rt * s.R;
-    const int e0 = te * s.TE;
-    const int ecount = (s.E - e0) < s.TE ? (s.E - e0) : s.TE;
-    const int rcount = (int)((s.batch - m0) < s.R ? (s.batch - m0) : s.R);
-    const int n_el = s.R * ecount;
-    const uint32_t mg = (1u << 22) / (uint32_t)ecount + 1u;
+__device__ __forceinline__ void cv_store(float *__restrict__ dst, const float *buf, const CvShape &s,
+                                         const CvTile &x, const int64_t *gb) {
 #pragma unroll 4
-    for (int idx = threadIdx.x; idx < n_el; idx += CV_THREADS) {
+    for (int idx = threadIdx.x; idx < x.n_el; idx += CV_THREADS) {
         if (DIR == 0) {
             const int r = idx & s.rmask, e = idx >> s.rshift;
-            if (r < rcount) dst[gb[r >> 5] + (int64_t)(e0 + e) * s.C + (r & 31)] = buf[r * s.ld + e];
+            if (r < x.rcount) dst[gb[r >> 5] + (int64_t)(x.e0 + e) * s.C + (r & 31)] = buf[r * s.ld + e];
         } else {
-            const int r = (int)(((uint64_t)idx * mg) >> 22), e = idx - r * ecount;
-            if (r < rcount) dst[(m0 + r) * s.E + e0 + e] = buf[r * s.ld + e];
+            const int r = (int)(((uint64_t)idx * x.mg) >> 22), e = idx - r * x.ecount;
+            if (r < x.rcount) dst[(x.m0 + r) * s.E + x.e0 + e] = buf[r * s.ld + e];
         }
     }
 }
 
+// Software pipeline in registers: the 16 loads of tile t+1 are issued before
+// tile t is written out, so loads stay in flight during the store phase.
 template <int DIR>
 __global__ void __launch_bounds__(CV_THREADS, 4)
 convert_kernel(const float *__restrict__ src, float *__restrict__ dst, CvShape s) {
-    extern __shared__ float smem[];                 // 2 x [R][ld]
+    extern __shared__ float buf[];                  // [R][ld]
     __shared__ int64_t gbase[2][CV_GMAX];
-    const size_t bsz = (size_t)s.R * s.ld;
-    auto buf = [&](int i) { return smem + i * bsz; };
     auto fill_gbase = [&](int slot, int64_t t) {
         const int64_t m0 = (t / s.elem_tiles) * s.R;
         for (int g = threadIdx.x; g < s.G; g += CV_THREADS) gbase[slot][g] = group_base(m0 + 32 * g, s.C, s.E);
     };
     int64_t t = blockIdx.x;
     if (t >= s.tiles) return;
+    float v[CV_PER];
+    int slot[CV_PER];
     fill_gbase(0, t);
     __syncthreads();
-    cv_issue_loads<DIR>(src, buf(0), s, t, gbase[0]);
-    cp_async_commit();
+    CvTile x = cv_tile(s, t);
+#pragma unroll
+    for (int k = 0; k < CV_PER; ++k) {
+        int64_t off;
+        slot[k] = -1;
+        if (cv_src<DIR>(s, x, gbase[0], threadIdx.x + k * CV_THREADS, slot[k], off)) v[k] = src[off];
+        else slot[k] = -1;
+    }
     int cur = 0;
     for (; t < s.tiles; t += gridDim.x) {
+#pragma unroll
+        for (int k = 0; k < CV_PER; ++k)
+            if (slot[k] >= 0) buf[slot[k]] = v[k];
         const int64_t tn = t + gridDim.x;
-        if (tn < s.tiles) {                         // prefetch the next tile into the other buffer
-            fill_gbase(cur ^ 1, tn);
-            __syncthreads();
-            cv_issue_loads<DIR>(src, buf(cur ^ 1), s, tn, gbase[cur ^ 1]);
+        const bool more = tn < s.tiles;
+        if (more) fill_gbase(cur ^ 1, tn);
+        __syncthreads();                            // tile t in smem, next gbase visible
+        if (more) {                                 // next tile's loads, in flight during the stores
+            const CvTile xn = cv_tile(s, tn);
+#pragma unroll
+            for (int k = 0; k < CV_PER; ++k) {
+                int64_t off;
+                if (cv_src<DIR>(s, xn, gbase[cur ^ 1], threadIdx.x + k * CV_THREADS, slot[k], off)) v[k] = src[off];
+                else slot[k] = -1;
+            }
         }
-        cp_async_commit();
-        cp_async_wait<1>();                         // tile t has landed (this thread's copies)
-        __syncthreads();                            // ... and everybody else's
-        cv_store<DIR>(dst, buf(cur), s, t, gbase[cur]);
-        __syncthreads();                            // buffer cur is free again
+        cv_store<DIR>(dst, buf, s, x, gbase[cur]);
+        __syncthreads();                            // buf and gbase[cur] free
+        if (more) x = cv_tile(s, tn);
         cur ^= 1;
     }
-    cp_async_wait<0>();
 }
 
 cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float *src, float *dst,
@@ -150,7 +167,7 @@ cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float
     while ((1 << s.rshift) < s.R) ++s.rshift;
     s.elem_tiles = (s.E + s.TE - 1) / s.TE;
     s.tiles = ((batch + s.R - 1) / s.R) * s.elem_tiles;
-    const size_t sm = 2 * (size_t)s.R * s.ld * sizeof(float);
+    const size_t sm = (size_t)s.R * s.ld * sizeof(float);
     int dev = 0, sms = 148, per_sm = 4;
     if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     if (dir == 0) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, convert_kernel<0>, CV_THREADS, sm);

@@ -72,6 +72,8 @@ template <int N, int NR, int CT>
 cudaError_t launch_potrs(const SolveArgs &a, int rhs0);
 template <int N, int NR, int CT>
 cudaError_t launch_sposv(const SolveArgs &a);
+template <int N, int CT, int S, bool TMA>
+cudaError_t launch_sposv_ptmem(const SolveArgs &a);
 
 // Grid size for one-thread-per-matrix kernels.
 inline unsigned grid_for(int64_t batch, int tpb) {

@@ -24,6 +24,7 @@
 
 #include "common.cuh"
 #include "launch.h"
+#include "potrs.cuh"
 #include "ptx.cuh"
 
 namespace bsp {
@@ -98,10 +99,17 @@ struct TmemShape {
     static_assert(CTM >= 1, "TMEM must hold at least one tile column");
 };
 
-template <int N, int CT, int S, bool TMA>
+// SOLVE: fused SPOSV with one right-hand side: B (n x 1 per
+// matrix, interleaved like A) is solved while every column of L is still on
+// chip -- forward substitution rides along the panel tile loop and the
+// register tail, backward substitution reads L back from TMEM / shared memory /
+// registers.  x lives in shared memory ([i][lane], after the panel part).  Op
+// order is potrs.cuh's, so X is bitwise identical to factor-then-SPOTRS.
+template <int N, int CT, int S, bool TMA, bool SOLVE = false>
 __global__ void __launch_bounds__(128, TmemShape<N, S>::COLS == 256 ? 2 : 1)
 potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
-                   int32_t *__restrict__ nfailed, int64_t batch, int64_t cs) {
+                   int32_t *__restrict__ nfailed, int64_t batch, int64_t cs,
+                   float *__restrict__ Bx = nullptr) {
     using SH = TmemShape<N, S>;
     constexpr int NB = 4, TR = SH::TR, TC = SH::TC, CTM = SH::CTM, CS = SH::CS;
     constexpr int NT = SH::NT, T = SH::T, PSM = SH::PSM;
@@ -117,7 +125,9 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
     const bool active = gid < batch;
     const int64_t g = active ? gid : batch - 1;
     const Addr<N, CT> ad(A, g, cs);
-    float *Q = smem + (size_t)warp * (PSM > 0 ? PSM : 1) * 32 + lane;   // lane-private view
+    constexpr int QW = (PSM > 0 ? PSM : 1) + (SOLVE ? N : 0);      // floats per lane per warp
+    float *Q = smem + (size_t)warp * QW * 32 + lane;                   // lane-private view
+    float *X = Q + (PSM > 0 ? PSM : 1) * 32;                           // x_i at X[i * 32]
     auto qs = [&](int m, int c) { return (c * N - (c * (c - 1)) / 2 + (m - c)) - SB0; };
 
     // ---- TMEM: warp 0 allocates 256 columns for the CTA ---------------------
@@ -148,7 +158,7 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                 const float *chunk = A + q * 32 * (N * N);
 #pragma unroll 1
                 for (int c = CS; c < S; ++c)
-                    bulk_g2s(smem + (size_t)warp * PSM * 32 + qs(c, c) * 32, chunk + (c + c * N) * 32,
+                    bulk_g2s(smem + (size_t)warp * QW * 32 + qs(c, c) * 32, chunk + (c + c * N) * 32,
                              (uint32_t)((N - c) * 32 * 4), &bars[warp]);
             }
         } else {
@@ -157,6 +167,13 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
 #pragma unroll 4
                 for (int m = c; m < N; ++m) cp_async4(Q + qs(m, c) * 32, ad.at(m, c));
         }
+    }
+
+    // ---- right-hand side -> shared memory (fused solve) ----------------------
+    if constexpr (SOLVE) {
+        const RectAddr<N, CT> ba(Bx, g, cs, 1);
+#pragma unroll 4
+        for (int i = 0; i < N; ++i) X[i * 32] = ld_stream(ba.at(i, 0));
     }
 
     // ---- trailing triangle -> registers ------------------------------------
@@ -275,6 +292,19 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
         float rinv[NB];
 #pragma unroll
         for (int k = 0; k < NB; ++k) rinv[k] = f_rcp(dg[k + k * NB]);
+        float xcb[NB];                                  // forward substitution, this block
+        if constexpr (SOLVE) {
+#pragma unroll
+            for (int k = 0; k < NB; ++k) xcb[k] = X[(CB * NB + k) * 32];
+#pragma unroll
+            for (int k = 0; k < NB; ++k) {
+                xcb[k] = f_mul(xcb[k], rinv[k]);
+#pragma unroll
+                for (int i = k + 1; i < NB; ++i) xcb[i] = f_upd(xcb[i], dg[i + k * NB], xcb[k]);
+            }
+#pragma unroll
+            for (int k = 0; k < NB; ++k) X[(CB * NB + k) * 32] = xcb[k];
+        }
         // (b) off-diagonal tiles (rb, CB), rb > CB: GEMM updates, then strsm_tile.
         //     ROWS = real rows of the tile row (4, or N % 4 for a ragged last one,
         //     peeled so the padded rows cost no arithmetic)
@@ -314,6 +344,17 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                         acc[i + j * NB] = f_upd(acc[i + j * NB], acc[i + k * NB], dg[j + k * NB]);
             }
             put_tile(rb, acc, cb_, FALSE_{});
+            if constexpr (SOLVE) {                      // x_rows -= L(rb, CB) x_CB, k ascending
+                float xr[NB];
+#pragma unroll
+                for (int i = 0; i < ROWS; ++i) xr[i] = X[(rb * NB + i) * 32];
+#pragma unroll
+                for (int k = 0; k < NB; ++k)
+#pragma unroll
+                    for (int i = 0; i < ROWS; ++i) xr[i] = f_upd(xr[i], acc[i + k * NB], xcb[k]);
+#pragma unroll
+                for (int i = 0; i < ROWS; ++i) X[(rb * NB + i) * 32] = xr[i];
+            }
         };
         constexpr int TRF = N / NB;                  // full tile rows
 #pragma unroll 1
@@ -370,7 +411,56 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
 #pragma unroll
             for (int m = k; m < NT; ++m) st_stream(ad.at(m + S, k + S), r[tri<NT>(m, k)]);
         }
+        if constexpr (SOLVE) {                          // forward step j = S + k
+            const float xk = f_mul(X[(S + k) * 32], inv);
+            X[(S + k) * 32] = xk;
+#pragma unroll
+            for (int i = k + 1; i < NT; ++i) X[(S + i) * 32] = f_upd(X[(S + i) * 32], r[tri<NT>(i, k)], xk);
+        }
     });
+    if constexpr (SOLVE) {
+        // backward substitution (dot form, j ascending), trailing rows from registers
+        sfor<0, NT>([&](auto t_) {
+            constexpr int i = NT - 1 - BSP_CI(t_);
+            float sacc = X[(S + i) * 32];
+#pragma unroll
+            for (int j = i + 1; j < NT; ++j) sacc = f_upd(sacc, r[tri<NT>(j, i)], X[(S + j) * 32]);
+            X[(S + i) * 32] = f_mul(sacc, f_rcp(r[tri<NT>(i, i)]));
+        });
+        // ... panel rows i = S-1..0: column i of L from TMEM tiles / shared memory
+#pragma unroll 1
+        for (int i = S - 1; i >= 0; --i) {
+            const int cb = i / NB, ii = i - cb * NB;
+            float sacc = X[i * 32];
+            float lii = 0.0f;
+#pragma unroll 1
+            for (int rb = cb; rb < TR; ++rb) {
+                float l[NB];
+                if (cb < CTM) {
+                    tmem_ld4(tbase + tidx(rb, cb) + (uint32_t)(ii * NB), l);
+                    tmem_wait_ld();
+                } else {
+#pragma unroll
+                    for (int q = 0; q < NB; ++q) {
+                        const int m = rb * NB + q;
+                        l[q] = (m < N && m >= i) ? Q[qs(m, i) * 32] : 0.0f;
+                    }
+                }
+                if (rb == cb) lii = l[ii];
+#pragma unroll
+                for (int q = 0; q < NB; ++q) {
+                    const int j = rb * NB + q;
+                    if (j > i && j < N) sacc = f_upd(sacc, l[q], X[j * 32]);
+                }
+            }
+            X[i * 32] = f_mul(sacc, f_rcp(lii));
+        }
+        if (active && inf == 0) {                       // SPOSV: failed matrices keep B
+            const RectAddr<N, CT> ba(Bx, g, cs, 1);
+#pragma unroll 4
+            for (int i = 0; i < N; ++i) st_stream(ba.at(i, 0), X[i * 32]);
+        }
+    }
     if (active) info[gid] = inf;
     count_failures(active && inf != 0, nfailed);
 
@@ -392,10 +482,24 @@ cudaError_t launch_ptmem(const FactorArgs &a) {
     size_t sm = (size_t)4 * SH::PSM * 32 * 4;
     const size_t floor_sm = SH::COLS == 256 ? 80 * 1024 : 120 * 1024;
     if (sm < floor_sm) sm = floor_sm;
-    auto kern = potrf_ptmem_kernel<N, CT, S, TMA>;
+    auto kern = potrf_ptmem_kernel<N, CT, S, TMA, false>;
     const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
-    kern<<<grid_for(a.batch, 128), 128, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
+    kern<<<grid_for(a.batch, 128), 128, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride,
+                                                         nullptr);
+    return cudaGetLastError();
+}
+
+template <int N, int CT, int S, bool TMA>
+cudaError_t launch_sposv_ptmem(const SolveArgs &a) {
+    using SH = TmemShape<N, S>;
+    size_t sm = (size_t)4 * ((SH::PSM > 0 ? SH::PSM : 1) + N) * 32 * 4;
+    const size_t floor_sm = SH::COLS == 256 ? 80 * 1024 : 120 * 1024;
+    if (sm < floor_sm) sm = floor_sm;
+    auto kern = potrf_ptmem_kernel<N, CT, S, TMA, true>;
+    const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e != cudaSuccess) return e;
+    kern<<<grid_for(a.batch, 128), 128, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride, a.B);
     return cudaGetLastError();
 }
 

@@ -52,7 +52,7 @@ def check_solution(n, nrhs, batch, chunk, A_c, B_c, Ai, Bi, Aout, Bout, info):
     return X
 
 
-@pytest.mark.parametrize("n", [1, 2, 5, 8, 13, 16, 20, 21, 24, 32, 33, 48, 64])
+@pytest.mark.parametrize("n", [1, 2, 5, 8, 13, 16, 20, 21, 24, 29, 32, 33, 40, 44, 48, 64])
 @pytest.mark.parametrize("nrhs", [1, 3, 5])
 @pytest.mark.parametrize("chunk", [32, 0])
 def test_sposv_matches_oracle(n, nrhs, chunk):
@@ -65,8 +65,9 @@ def test_sposv_matches_oracle(n, nrhs, chunk):
     assert cnt == int((info != 0).sum()) > 0
 
 
-@pytest.mark.parametrize("n", [3, 8, 16, 20])
-@pytest.mark.parametrize("nrhs", [1, 2, 4])
+@pytest.mark.parametrize("n,nrhs", [(3, 1), (3, 4), (8, 2), (16, 1), (16, 4), (20, 3),
+                                    (24, 1), (25, 1), (28, 1), (31, 1), (32, 1), (33, 1), (36, 1),
+                                    (40, 1), (44, 1)])
 def test_fused_equals_factor_then_solve_bitwise(n, nrhs):
     batch = 300
     b = np.arange(batch, dtype=np.uint64)
