@@ -32,7 +32,7 @@ def timed(fn, prep, reps=5):
     return statistics.median(ts)
 
 
-for n in (4, 8, 16, 20, 24, 32):
+for n in (4, 8, 16, 20, 24, 28, 32, 36, 40, 44):
     for nrhs in (1, 4):
         A = torch.empty(bsp.batch_interleaved_elems(n, B, chunk), device="cuda")
         A0 = torch.empty_like(A)
@@ -49,7 +49,7 @@ for n in (4, 8, 16, 20, 24, 32):
         r = dict(n=n, nrhs=nrhs, sposv_ms=round(t_sposv, 4), potrs_ms=round(t_potrs, 4),
                  sposv_gbs=round(B * (fb + rb) / t_sposv / 1e6, 1),
                  potrs_gbs=round(B * (2 * 2 * n * (n + 1) + rb) / t_potrs / 1e6, 1),
-                 fused=bool(n <= 20 and nrhs <= 4))
+                 fused=bool((n <= 20 and nrhs <= 4) or (24 <= n <= 44 and nrhs == 1)))
         rows.append(r)
         print(json.dumps(r), flush=True)
         del A, A0, Bm, B0
