@@ -447,14 +447,24 @@ def run_ours(a, w):
         slab = max(chunk or 32, ((32 << 20) // (2 * n * (n + 1))) // (chunk or 32) * (chunk or 32))
         t_pipe = e2e_run(slab)                      # the copy pipeline, for comparison
         gfl = lambda t: round(Btot * flops_per_matrix(n) / t / 1e9, 3)
-        e2e = {"value": gfl(t_zero), "unit": "Gflop/s", "h2d_bytes_per_step": hb,
-               "d2h_bytes_per_step": hb + 4 * B + 4, "ms_per_step": round(t_zero * 1e3, 3),
-               "path": "batch_spotrf_interleaved_host(slab=0) on pinned host interleaved storage: "
-                       "zero-copy, the factorization kernel reads/writes host memory over PCIe",
-               "pcie_gbs_each_way": round(hb / t_zero / 1e9, 2),
-               "copy_pipeline": {"value": gfl(t_pipe), "ms_per_step": round(t_pipe * 1e3, 3),
-                                 "slab_matrices": slab,
-                                 "path": "3-stream slab pipeline, lower-triangle 2-D copies"}}
+        # Both are the same public call (batch_spotrf_interleaved_host) on the same
+        # pinned buffers; slab selects the path.  Zero-copy throughput depends on the
+        # host's PCIe/coherence behaviour (measured 2.4-38 GB/s at n=16 on different
+        # boxes), the copy pipeline is steady: report the faster, keep both.
+        paths = {"zero_copy": {"value": gfl(t_zero), "ms_per_step": round(t_zero * 1e3, 3), "slab": 0,
+                               "path": "batch_spotrf_interleaved_host(slab=0) on pinned host interleaved "
+                                       "storage: zero-copy, the factorization kernel reads/writes host "
+                                       "memory over PCIe"},
+                 "copy_pipeline": {"value": gfl(t_pipe), "ms_per_step": round(t_pipe * 1e3, 3),
+                                   "slab": slab,
+                                   "path": f"batch_spotrf_interleaved_host(slab={slab}): 3-stream slab "
+                                           "pipeline, lower-triangle 2-D copies H2D / kernel / D2H"}}
+        best = "zero_copy" if t_zero <= t_pipe else "copy_pipeline"
+        tb = min(t_zero, t_pipe)
+        e2e = {"value": gfl(tb), "unit": "Gflop/s", "h2d_bytes_per_step": hb,
+               "d2h_bytes_per_step": hb + 4 * B + 4, "ms_per_step": round(tb * 1e3, 3),
+               "path": paths[best]["path"], "pcie_gbs_each_way": round(hb / tb / 1e9, 2),
+               "paths": paths}
 
     cpu = None
     if rank == 0 and world == 1 and not a.no_cpu_baseline:

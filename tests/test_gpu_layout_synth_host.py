@@ -14,9 +14,12 @@ pytestmark = pytest.mark.gpu
 
 @pytest.mark.parametrize("n", [1, 2, 3, 5, 8, 16, 31, 32, 64])
 @pytest.mark.parametrize("chunk", [32, 64, 0, 160])
-def test_conversion_matches_layout_definition(n, chunk):
+@pytest.mark.parametrize("batch", [517, 1024, 96, 1])
+def test_conversion_matches_layout_definition(n, chunk, batch):
+    """batch 517: ragged last group (32-bit interleaved accesses, masked); 1024 and
+    96 with chunk 0: C % 4 == 0 (128-bit interleaved path); even n: 128-bit
+    canonical path; odd n: 32-bit canonical path (rows not 16-B aligned)."""
     torch = torch_mod()
-    batch = 517
     rng = np.random.default_rng(n * 1000 + chunk)
     canon = rng.standard_normal((batch, n * n)).astype(np.float32)
     expect = layout.to_interleaved(n, chunk, canon, fill_bits=synth.PAD_BITS)
