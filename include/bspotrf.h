@@ -66,10 +66,18 @@ enum {
     BSPOTRF_VARIANT_RTMA = 6, /* REG with TMA bulk copies in and out of a
                                  shared-memory image (chunk 32 only); `param`
                                  warps per CTA (2 or 4); 4 <= n <= 20         */
-    BSPOTRF_VARIANT_RTMAP = 7 /* persistent RTMA: each warp loops over chunks,
+    BSPOTRF_VARIANT_RTMAP = 7, /* persistent RTMA: each warp loops over chunks,
                                  the next chunk's TMA load overlapping this
                                  chunk's arithmetic; per-thread stores; grid =
                                  resident warps; chunk 32; 4 <= n <= 20       */
+    BSPOTRF_VARIANT_QTM = 8   /* `param` (4 or 8) threads per matrix, each
+                                 owning tile rows; the whole matrix on chip
+                                 (off-diagonal 4x4 tiles in Tensor Memory and
+                                 shared memory), left-looking; staging 1 =
+                                 256 TMEM columns per CTA (two CTAs per SM),
+                                 0/2 = 512 (one), input streamed by cp.async;
+                                 3/4 = the same with the input preloaded;
+                                 any chunk; 33 <= n <= 64                     */
 };
 
 /* Launch tuning (a row of the autotuning table). */

@@ -50,6 +50,12 @@ cudaError_t launch_regtma(const FactorArgs &a);
 template <int N, int W>
 cudaError_t launch_rtmap(const FactorArgs &a);
 
+// Variant QTM: P threads per matrix, the whole matrix on chip (TMEM + shared
+// memory), COLS TMEM columns per 128-thread CTA, input streamed (PRE = false)
+// or preloaded (csrc/potrf_qtm.cuh).
+template <int N, int CT, int P, int COLS, bool PRE>
+cudaError_t launch_qtm(const FactorArgs &a);
+
 // Variant TILE: the paper's top-looking tile algorithm, NB x NB register
 // tiles streamed from global memory, runtime chunk stride (csrc/potrf_tile.cuh).
 template <int N, int NB>

@@ -9,6 +9,8 @@ Exhaustive over the B200 axes (north star (4)):
             TMA bulk copy (staging 1) or per-thread cp.async (staging 2)
       TILE  tile ops unrolled, outer loops rolled, NB x NB tiles
             (paper: partially unrolled top-looking, n_b = NB)
+      PANEL/PTMEM/RTMA/RTMAP  see include/bspotrf.h
+      QTM   P threads per matrix (4, 8), TMEM columns per CTA (256, 512), n > 32
   * threads per block       -- 32..256
 Each point: regenerate the batch in place (device generator), flush L2, time
 ONE launch with CUDA events; median of --reps.  Every point is also checked
@@ -85,6 +87,13 @@ def candidates(n, chunk):
                 c.append(dict(variant=SMEM, threads_per_block=0, param=s, staging=1))
             for tpb in (32, 64, 128):
                 c.append(dict(variant=SMEM, threads_per_block=tpb, param=s, staging=2))
+    if 33 <= n <= 64:
+        sys.path.insert(0, os.path.join(ROOT, "scripts"))
+        import gen_instances
+        for p_, cols, pre in gen_instances.QTM_COMBOS:
+            if gen_instances.qtm_fits(n, p_, cols, pre):
+                c.append(dict(variant=bsp.VARIANT_QTM, threads_per_block=128, param=p_,
+                              staging=gen_instances.qtm_staging(cols, pre)))
     for nb in (2, 4, 8):
         if nb <= n or nb == 2:
             for tpb in (64, 128, 256):
@@ -102,7 +111,7 @@ def main():
     ap.add_argument("--kind", default="dd")
     ap.add_argument("--skip-from", action="append", default=[],
                     help="JSONL files whose points are already measured")
-    ap.add_argument("--variants", default="1,2,3,4,5,6,7")
+    ap.add_argument("--variants", default="1,2,3,4,5,6,7,8")
     a = ap.parse_args()
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     done = set()

@@ -27,16 +27,17 @@ for n in ns:
         if (n, c) in best:
             entries.append(dict(n=n, chunk=c, **key(best[(n, c)])))
     # any other chunk: runtime-stride-capable best at 256 (else 32 w/o TMA)
-    cand = [r for r in ok if r["n"] == n and r["chunk"] in (256, 512) and r["staging"] != 1]
+    tma = lambda r: r["staging"] == 1 and r["variant"] != 8        # QTM staging 1 is not TMA
+    cand = [r for r in ok if r["n"] == n and r["chunk"] in (256, 512) and not tma(r)]
     if not cand:
-        cand = [r for r in ok if r["n"] == n and r["staging"] != 1]
+        cand = [r for r in ok if r["n"] == n and not tma(r)]
     if cand:
         b = min(cand, key=lambda r: r["ms"])
         entries.append(dict(n=n, chunk=-1, **key(b)))
 json.dump({"source": f"B200 autotune sweep {src}", "entries": entries}, open(out_table, "w"), indent=1)
 print(f"{len(entries)} rows -> {out_table}")
 if out_md:
-    V = {1: "REG", 2: "SMEM", 3: "TILE", 4: "PANEL", 5: "PTMEM", 6: "RTMA", 7: "RTMAP"}
+    V = {1: "REG", 2: "SMEM", 3: "TILE", 4: "PANEL", 5: "PTMEM", 6: "RTMA", 7: "RTMAP", 8: "QTM"}
     with open(out_md, "w") as f:
         f.write("| n | best chunk | variant | tpb | param | staging | ms (1M) | GB/s | Gflop/s | "
                 "best chunk=0 GB/s | 32 | 64 | 128 | 256 | 512 |\n|---|---|---|---|---|---|---|---|---|---|---|---|---|---|---|\n")

@@ -71,6 +71,41 @@ def _ptmem_s(n):
     return gen_instances.ptmem_s_values(n)
 
 
+def gen_instances_mod():
+    import sys, os
+    sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(__file__)), "scripts"))
+    import gen_instances
+    return gen_instances
+
+
+def _qtm_combos(n):
+    import sys, os
+    sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(__file__)), "scripts"))
+    import gen_instances
+    if n not in gen_instances.QTM_N:
+        return []
+    return [(p_, c, pre) for p_, c, pre in gen_instances.QTM_COMBOS if gen_instances.qtm_fits(n, p_, c, pre)]
+
+
+@pytest.mark.parametrize("n", [33, 35, 38, 44, 45, 47, 50, 53, 57, 60, 62, 64])
+@pytest.mark.parametrize("chunk", [32, 0, 96])
+def test_qtm_parity_failures_ragged(n, chunk):
+    """Variant QTM (P threads per matrix, matrix on chip): every (P, TMEM
+    columns) instance against the oracle, with injected failures, a batch that
+    is not a multiple of the matrices per CTA, and the runtime-stride path."""
+    batch = 3 * 32 + 13
+    canon, inter = make_batch(n, batch, chunk, kind="dd", seed=n, fail_seed=2018, fail_period=5)
+    failed, kk = synth.fail_plan(n, 2018, 5, np.arange(batch, dtype=np.uint64))
+    combos = _qtm_combos(n)
+    assert combos
+    for p_, cols, pre in combos:
+        t = dict(variant=bsp.VARIANT_QTM, threads_per_block=128, param=p_,
+                 staging=gen_instances_mod().qtm_staging(cols, pre))
+        out, info, cnt = run_gpu(n, batch, chunk, inter, tune=t)
+        assert np.array_equal(info, np.where(failed, kk + 1, 0)), t
+        assert_parity(n, batch, chunk, canon, inter, out, info, cnt)
+
+
 def _tunings(n, chunk):
     out = []
     if n <= 24:
@@ -92,6 +127,9 @@ def _tunings(n, chunk):
             out.append(dict(variant=bsp.VARIANT_PTMEM, threads_per_block=128, param=s, staging=2))
             if chunk == 32:
                 out.append(dict(variant=bsp.VARIANT_PTMEM, threads_per_block=128, param=s, staging=1))
+    for p_, cols, pre in _qtm_combos(n):
+        out.append(dict(variant=bsp.VARIANT_QTM, threads_per_block=128, param=p_,
+                        staging=gen_instances_mod().qtm_staging(cols, pre)))
     for tpb in (64, 256):
         for nb in (2, 4, 8):
             if nb <= n or nb == 2:
@@ -107,7 +145,7 @@ def _tunings(n, chunk):
 
 
 @pytest.mark.parametrize("n", [2, 7, 13, 16, 19, 20, 21, 23, 24, 25, 27, 28, 29, 30, 31, 32, 33, 36, 39,
-                               40, 44, 45, 64])
+                               40, 44, 45, 49, 56, 61, 64])
 @pytest.mark.parametrize("chunk", [32, 64, 0])
 def test_all_variants_bitwise_identical(n, chunk):
     """P8: every variant / staging / block size gives the same bits."""
