@@ -61,8 +61,9 @@ enum {
                                  SYRK, unrolled register tail; 20 <= n <= 32   */
     BSPOTRF_VARIANT_PTMEM = 5, /* PANEL with the first panel tile columns held in
                                  Tensor Memory (tcgen05.ld/st), 128-thread
-                                 CTAs with 256 TMEM columns each (two per SM);
-                                 TMA staging needs chunk 32; 24 <= n <= 32    */
+                                 CTAs with 256 TMEM columns each (two per SM;
+                                 512, one per SM, for n > 32); TMA staging
+                                 needs chunk 32; 24 <= n <= 44               */
     BSPOTRF_VARIANT_RTMA = 6, /* REG with TMA bulk copies in and out of a
                                  shared-memory image (chunk 32 only); `param`
                                  warps per CTA (2 or 4); 4 <= n <= 20         */
@@ -70,7 +71,7 @@ enum {
                                  the next chunk's TMA load overlapping this
                                  chunk's arithmetic; per-thread stores; grid =
                                  resident warps; chunk 32; 4 <= n <= 20       */
-    BSPOTRF_VARIANT_QTM = 8   /* `param` (4 or 8) threads per matrix, each
+    BSPOTRF_VARIANT_QTM = 8,  /* `param` (4 or 8) threads per matrix, each
                                  owning tile rows; the whole matrix on chip
                                  (off-diagonal 4x4 tiles in Tensor Memory and
                                  shared memory), left-looking; staging 1 =
@@ -78,6 +79,12 @@ enum {
                                  0/2 = 512 (one), input streamed by cp.async;
                                  3/4 = the same with the input preloaded;
                                  any chunk; 33 <= n <= 64                     */
+    BSPOTRF_VARIANT_REGX = 9  /* REG with the extra sweep axes: `param` (1, 2,
+                                 4) matrices per thread; staging 1 = fast-math
+                                 sqrt/rcp (sqrt.approx, rcp.approx, ftz;
+                                 tolerance-checked, not bitwise reproducible,
+                                 never chosen by the default table), 0 = IEEE;
+                                 <= 128 threads per block; 1 <= n <= 16       */
 };
 
 /* Launch tuning (a row of the autotuning table). */

@@ -122,6 +122,8 @@ static LaunchFn resolve(int n, int chunk, const bspotrf_tuning &t, int *tpb_out)
         return chunk == 32 ? find(t.variant, n, t.param, 32, 1) : nullptr;
     case BSPOTRF_VARIANT_TILE:
         return find(BSPOTRF_VARIANT_TILE, n, t.param, 0, 0);
+    case BSPOTRF_VARIANT_REGX:
+        return find(BSPOTRF_VARIANT_REGX, n, t.param, 0, t.staging == 1 ? 1 : 0);
     case BSPOTRF_VARIANT_QTM: {
         *tpb_out = 128;
         const int st = t.staging == 0 ? 2 : t.staging;   // 1/2: 256/512 TMEM columns, streamed;

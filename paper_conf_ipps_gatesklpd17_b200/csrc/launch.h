@@ -50,6 +50,11 @@ cudaError_t launch_regtma(const FactorArgs &a);
 template <int N, int W>
 cudaError_t launch_rtmap(const FactorArgs &a);
 
+// Variant REGX: REG with M matrices per thread and optional fast-math sqrt/rcp
+// (csrc/potrf_reg.cuh).
+template <int N, int M, bool FAST>
+cudaError_t launch_regx(const FactorArgs &a);
+
 // Variant QTM: P threads per matrix, the whole matrix on chip (TMEM + shared
 // memory), COLS TMEM columns per 128-thread CTA, input streamed (PRE = false)
 // or preloaded (csrc/potrf_qtm.cuh).

@@ -87,6 +87,12 @@ def candidates(n, chunk):
                 c.append(dict(variant=SMEM, threads_per_block=0, param=s, staging=1))
             for tpb in (32, 64, 128):
                 c.append(dict(variant=SMEM, threads_per_block=tpb, param=s, staging=2))
+    if n <= 16:
+        sys.path.insert(0, os.path.join(ROOT, "scripts"))
+        import gen_instances
+        for m, fast in gen_instances.regx_combos(n):
+            for tpb in (64, 128):
+                c.append(dict(variant=bsp.VARIANT_REGX, threads_per_block=tpb, param=m, staging=int(fast)))
     if 33 <= n <= 64:
         sys.path.insert(0, os.path.join(ROOT, "scripts"))
         import gen_instances
@@ -111,7 +117,7 @@ def main():
     ap.add_argument("--kind", default="dd")
     ap.add_argument("--skip-from", action="append", default=[],
                     help="JSONL files whose points are already measured")
-    ap.add_argument("--variants", default="1,2,3,4,5,6,7,8")
+    ap.add_argument("--variants", default="1,2,3,4,5,6,7,8")   # 9 (REGX) on request
     a = ap.parse_args()
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     done = set()

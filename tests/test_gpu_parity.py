@@ -106,6 +106,23 @@ def test_qtm_parity_failures_ragged(n, chunk):
         assert_parity(n, batch, chunk, canon, inter, out, info, cnt)
 
 
+@pytest.mark.parametrize("n", [1, 2, 3, 5, 8, 11, 12, 16])
+@pytest.mark.parametrize("chunk", [32, 0, 96])
+def test_regx_multi_matrix_and_fast_math(n, chunk):
+    """Variant REGX: M matrices per thread (IEEE: bitwise equal to
+    the Fig. 9 emulator) and the fast-math form (reading R4: O1-O4 only, exempt from
+    the bitwise pins), with injected failures and a ragged batch."""
+    batch = 2 * 128 * 4 + 77
+    canon, inter = make_batch(n, batch, chunk, kind="als", seed=n + 3, fail_seed=2018, fail_period=9)
+    failed, kk = synth.fail_plan(n, 2018, 9, np.arange(batch, dtype=np.uint64))
+    for m, fast in gen_instances_mod().regx_combos(n):
+        for tpb in (64, 128):
+            t = dict(variant=bsp.VARIANT_REGX, threads_per_block=tpb, param=m, staging=int(fast))
+            out, info, cnt = run_gpu(n, batch, chunk, inter, tune=t)
+            assert np.array_equal(info, np.where(failed, kk + 1, 0)), t
+            assert_parity(n, batch, chunk, canon, inter, out, info, cnt, emulate=not fast)
+
+
 def _tunings(n, chunk):
     out = []
     if n <= 24:
@@ -127,6 +144,9 @@ def _tunings(n, chunk):
             out.append(dict(variant=bsp.VARIANT_PTMEM, threads_per_block=128, param=s, staging=2))
             if chunk == 32:
                 out.append(dict(variant=bsp.VARIANT_PTMEM, threads_per_block=128, param=s, staging=1))
+    for m, fast in gen_instances_mod().regx_combos(n) if n in gen_instances_mod().REGX_N else []:
+        if not fast:                              # IEEE: same op sequence -> same bits
+            out.append(dict(variant=bsp.VARIANT_REGX, threads_per_block=128, param=m, staging=0))
     for p_, cols, pre in _qtm_combos(n):
         out.append(dict(variant=bsp.VARIANT_QTM, threads_per_block=128, param=p_,
                         staging=gen_instances_mod().qtm_staging(cols, pre)))
