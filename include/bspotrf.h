@@ -79,12 +79,18 @@ enum {
                                  0/2 = 512 (one), input streamed by cp.async;
                                  3/4 = the same with the input preloaded;
                                  any chunk; 33 <= n <= 64                     */
-    BSPOTRF_VARIANT_REGX = 9  /* REG with the extra sweep axes: `param` (1, 2,
+    BSPOTRF_VARIANT_REGX = 9, /* REG with the extra sweep axes: `param` (1, 2,
                                  4) matrices per thread; staging 1 = fast-math
                                  sqrt/rcp (sqrt.approx, rcp.approx, ftz;
                                  tolerance-checked, not bitwise reproducible,
                                  never chosen by the default table), 0 = IEEE;
                                  <= 128 threads per block; 1 <= n <= 16       */
+    BSPOTRF_VARIANT_RCW = 10  /* row-cyclic warps: 8 warps share 32 matrices
+                                 (lane = matrix), warp h owns rows 8r+h, the
+                                 factor in Tensor Memory, left-looking over
+                                 8-wide column blocks; `param` = CTAs per SM
+                                 (1: 512 TMEM columns, any n; 2: 256 each,
+                                 n <= 48); any chunk; 33 <= n <= 64           */
 };
 
 /* Launch tuning (a row of the autotuning table). */

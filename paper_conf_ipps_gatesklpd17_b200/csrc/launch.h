@@ -61,6 +61,11 @@ cudaError_t launch_regx(const FactorArgs &a);
 template <int N, int CT, int P, int COLS, bool PRE>
 cudaError_t launch_qtm(const FactorArgs &a);
 
+// Variant RCW: 8 warps share 32 matrices (lane = matrix, warp h owns rows
+// 8r+h), factor in TMEM, NCTA CTAs per SM (csrc/potrf_rcw.cuh).
+template <int N, int CT, int NCTA>
+cudaError_t launch_rcw(const FactorArgs &a);
+
 // Variant TILE: the paper's top-looking tile algorithm, NB x NB register
 // tiles streamed from global memory, runtime chunk stride (csrc/potrf_tile.cuh).
 template <int N, int NB>

@@ -1,0 +1,237 @@
+// potrf_rcw.cuh -- variant RCW ("row-cyclic warps"): eight warps share 32
+// matrices, lane = matrix, warp h owns the rows i = 8r + h (r = 0..R-1) of all
+// 32; the factor stays on chip in Tensor Memory.  For 33 <= n <= 64 (SURVEY
+// §8(f) f2), where one thread per matrix no longer fits on chip.
+//
+// Why this shape.  At n = 64 the lower triangle is 2080 floats; 32 matrices
+// need 266 KB, which only TMEM (256 KB) + shared memory can hold -- one CTA
+// per SM.  QTM (P = 4 threads per matrix inside one warp) gets there with 4
+// warps per SM, rows of different length in one warp instruction (dead lanes:
+// 28% of its FFMAs) and a per-column publish through TMEM round trips.  Here:
+//   * a warp instruction touches the SAME element (i, j) of 32 consecutive
+//     matrices: every global access is one 128-B line, and every lane of a
+//     warp does the same work (no dead lanes, uniform branches only);
+//   * 8 warps per CTA (2 per scheduler) instead of 4;
+//   * warp h's rows live in TMEM (lane quarter h % 4, column half h / 4):
+//     slot r holds L(8r+h, 0..8r-1) at columns 4r(r-1) .. -- 224 columns at
+//     n = 64, so the whole factor fits in one 512-column allocation;
+//   * left-looking over 8-wide column blocks c: the rows 8c..8c+7 of L (the
+//     "b" operand every warp needs) are published to a row buffer RB(c) in
+//     shared memory by their owners while those owners stream them out of TMEM
+//     for their own GEMM in block c-1 (no extra TMEM reads);
+//   * the input streams in one block ahead (cp.async, each thread copies the
+//     elements it will read itself, so only its own completion is awaited).
+//     Shared memory is two halves of R units of 8 KB; in block c the half
+//     c % 2 holds RB(c) in units 0..c-1 and the input stage of block c in
+//     units c..R-1, the other half receives RB(c+1) and stage(c+1): exactly
+//     16 units at any time (RB grows as the stage shrinks).
+// Op order per element (i, j): fma with k = 0, 1, ..., j-1 ascending (GEMM over
+// k < 8c, then the in-block triangular updates), then mul by rcp.rn(L_jj) --
+// the Fig. 9 sequence of every other variant, so the output is bitwise
+// identical to REG/PTMEM/QTM (pin P8).
+#pragma once
+
+#include "common.cuh"
+#include "launch.h"
+#include "ptx.cuh"
+#include "potrf_tmem.cuh"
+
+namespace bsp {
+
+__device__ __forceinline__ void tmem_st8(uint32_t taddr, const float *v) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"r"(taddr),
+                 "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7])
+                 : "memory");
+}
+
+template <int N, int NCTA>
+struct RcwShape {
+    static constexpr int W = 8;                          // column-block width = warps per CTA
+    static constexpr int R = (N + W - 1) / W;            // row slots per warp (= column blocks)
+    static constexpr int COLS = NCTA == 1 ? 512 : 256;   // TMEM columns per CTA
+    static constexpr int HALF = COLS / 2;                // per warp (warps h and h+4 share lanes)
+    static constexpr int UNIT = W * W * 32;              // floats per 8 KB unit
+    __host__ __device__ static constexpr int off(int r) { return 4 * r * (r - 1); }
+    __host__ __device__ static constexpr int dt(int m, int k) { return m * (m + 1) / 2 + k; }
+    static constexpr size_t SMEM = (size_t)(2 * R * UNIT + 36 * 32) * sizeof(float);
+    static_assert(off(R) <= HALF, "slots exceed the TMEM column budget");
+};
+
+template <int N, int CT, int NCTA>
+__global__ void __launch_bounds__(256, NCTA)
+potrf_rcw_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__restrict__ nfailed,
+                 int64_t batch, int64_t cs) {
+    using SH = RcwShape<N, NCTA>;
+    constexpr int R = SH::R, UNIT = SH::UNIT;
+    extern __shared__ __align__(16) float smf[];
+    __shared__ uint32_t tmem_base_sh;
+
+    const int h = threadIdx.x >> 5, q = threadIdx.x & 31;
+    const int64_t gm = (int64_t)blockIdx.x * 32 + q;
+    const bool active = gm < batch;
+    const Addr<N, CT> ad(A, active ? gm : batch - 1, cs);
+    float *DB = smf + 2 * R * UNIT;                      // diagonal block gather [36][32]
+    auto unit = [&](int half, int u) { return smf + (size_t)(half * R + u) * UNIT; };
+
+    if (h == 0) {
+        tmem_alloc(&tmem_base_sh, SH::COLS);
+        tmem_relinquish();
+    }
+    tmem_fence_before();
+    __syncthreads();
+    tmem_fence_after();
+    const uint32_t tb = tmem_base_sh + ((uint32_t)(32 * (h & 3)) << 16) + (uint32_t)((h >> 2) * SH::HALF);
+
+    // input of column block c -> stage units c..R-1 of half c % 2: element
+    // (8r+h, 8c+w) at [w][h][q] of unit r; only my own rows, lower part only
+    auto prefetch = [&](auto c_) {
+        constexpr int c = BSP_CI(c_);
+        sfor<c, R>([&](auto r_) {
+            constexpr int r = BSP_CI(r_);
+            const int i = 8 * r + h;
+            if (i < N) {
+                float *dst = unit(c & 1, r) + h * 32 + q;
+#pragma unroll
+                for (int w = 0; w < 8; ++w)
+                    if (8 * c + w < N && (r > c || w <= h)) cp_async4(dst + w * 256, ad.at(i, 8 * c + w));
+            }
+        });
+        cp_async_commit();
+    };
+    prefetch(std::integral_constant<int, 0>{});
+
+    int inf = 0;
+    float acc[R][8];
+    sfor<0, R>([&](auto c_) {
+        constexpr int c = BSP_CI(c_);
+        cp_async_wait<0>();                              // my stage(c) copies landed
+        __syncthreads();                                 // RB(c) published; old units free
+        if constexpr (c + 1 < R) prefetch(std::integral_constant<int, c + 1>{});
+
+        // (a) accumulators of my live rows = A(8r+h, 8c..8c+7)
+        sfor<c, R>([&](auto r_) {
+            constexpr int r = BSP_CI(r_);
+            const float *src = unit(c & 1, r) + h * 32 + q;
+#pragma unroll
+            for (int w = 0; w < 8; ++w)
+                acc[r][w] = (r > c || w <= h) && 8 * c + w < N ? src[w * 256] : 0.0f;
+        });
+
+        // (b) acc(r) -= L(8r+h, 0..8c-1) L(8c..8c+7, 0..8c-1)^T, k ascending; the
+        //     rows of block c+1 (my slot c+1) are published to RB(c+1) on the way
+        if constexpr (c > 0) {
+            const float4 *rb = reinterpret_cast<const float4 *>(unit(c & 1, 0)) + q;
+            float4 *rbn = reinterpret_cast<float4 *>(unit((c + 1) & 1, 0)) + h * 32 + q;
+#pragma unroll 1
+            for (int kq = 0; kq < 2 * c; ++kq) {
+                float b[8][4];
+#pragma unroll
+                for (int w = 0; w < 8; ++w) {
+                    const float4 x = rb[(kq * 8 + w) * 32];
+                    b[w][0] = x.x, b[w][1] = x.y, b[w][2] = x.z, b[w][3] = x.w;
+                }
+                float a[R][4];
+                sfor<c, R>([&](auto r_) {
+                    constexpr int r = BSP_CI(r_);
+                    tmem_ld4(tb + (uint32_t)(SH::off(r) + 4 * kq), a[r]);
+                });
+                tmem_wait_ld();
+                if constexpr (c + 1 < R) rbn[kq * 256] = make_float4(a[c + 1][0], a[c + 1][1], a[c + 1][2], a[c + 1][3]);
+                sfor<c, R>([&](auto r_) {
+                    constexpr int r = BSP_CI(r_);
+#pragma unroll
+                    for (int kk = 0; kk < 4; ++kk)
+#pragma unroll
+                        for (int w = 0; w < 8; ++w) acc[r][w] = f_upd(acc[r][w], a[r][kk], b[w][kk]);
+                });
+            }
+        }
+
+        // (c) diagonal block: gather rows 8c..8c+7, factor it in every warp (identical bits)
+#pragma unroll
+        for (int m = 0; m < 8; ++m)
+            if (m == h && 8 * c + m < N) {
+#pragma unroll
+                for (int w = 0; w <= m; ++w) DB[SH::dt(m, w) * 32 + q] = acc[c][w];
+            }
+        __syncthreads();
+        float d[36], inv[8];
+#pragma unroll
+        for (int t = 0; t < 36; ++t) d[t] = DB[t * 32 + q];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            if (8 * c + k >= N) break;
+            const float p = d[SH::dt(k, k)];
+            pivot_check(p, 8 * c + k, inf);
+            const float s = f_sqrt(p);
+            d[SH::dt(k, k)] = s;
+            inv[k] = f_rcp(s);
+#pragma unroll
+            for (int m = k + 1; m < 8; ++m) d[SH::dt(m, k)] = f_mul(d[SH::dt(m, k)], inv[k]);
+#pragma unroll
+            for (int j = k + 1; j < 8; ++j)
+#pragma unroll
+                for (int m = j; m < 8; ++m) d[SH::dt(m, j)] = f_upd(d[SH::dt(m, j)], d[SH::dt(m, k)], d[SH::dt(j, k)]);
+        }
+        if (active) {
+#pragma unroll
+            for (int m = 0; m < 8; ++m)
+                if (m == h && 8 * c + m < N) {
+#pragma unroll
+                    for (int w = 0; w <= m; ++w) st_stream(ad.at(8 * c + m, 8 * c + w), d[SH::dt(m, w)]);
+                }
+        }
+
+        // (d) triangular solve of my rows below the block; HBM, TMEM, RB(c+1)
+        sfor<c + 1, R>([&](auto r_) {
+            constexpr int r = BSP_CI(r_);
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+                if (8 * c + k >= N) break;
+                acc[r][k] = f_mul(acc[r][k], inv[k]);
+#pragma unroll
+                for (int j = k + 1; j < 8; ++j) acc[r][j] = f_upd(acc[r][j], acc[r][k], d[SH::dt(j, k)]);
+            }
+            const int i = 8 * r + h;
+            if (active && i < N) {
+#pragma unroll
+                for (int w = 0; w < 8; ++w)
+                    if (8 * c + w < N) st_stream(ad.at(i, 8 * c + w), acc[r][w]);
+            }
+            tmem_st8(tb + (uint32_t)(SH::off(r) + 8 * c), acc[r]);
+            if constexpr (r == c + 1) {
+                float4 *rbn = reinterpret_cast<float4 *>(unit((c + 1) & 1, 0)) + h * 32 + q;
+                rbn[(2 * c) * 256] = make_float4(acc[r][0], acc[r][1], acc[r][2], acc[r][3]);
+                rbn[(2 * c + 1) * 256] = make_float4(acc[r][4], acc[r][5], acc[r][6], acc[r][7]);
+            }
+        });
+        tmem_wait_st();
+    });
+
+    if (active && h == 0) info[gm] = inf;
+    if (h == 0) count_failures(active && inf != 0, nfailed);
+
+    tmem_fence_before();
+    __syncthreads();
+    if (h == 0) {
+        tmem_fence_after();
+        tmem_dealloc(tmem_base_sh, SH::COLS);
+    }
+}
+
+template <int N, int CT, int NCTA>
+cudaError_t launch_rcw(const FactorArgs &a) {
+    using SH = RcwShape<N, NCTA>;
+    auto kern = potrf_rcw_kernel<N, CT, NCTA>;
+    // one CTA per SM must own all 512 TMEM columns: ask for enough shared memory
+    // that a second CTA never becomes resident (it would spin in tcgen05.alloc)
+    size_t sm = SH::SMEM;
+    if constexpr (NCTA == 1)
+        if (sm < (size_t)116 * 1024) sm = (size_t)116 * 1024;
+    const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e != cudaSuccess) return e;
+    kern<<<grid_for(a.batch, 32), 256, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
+    return cudaGetLastError();
+}
+
+}  // namespace bsp

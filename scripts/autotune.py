@@ -11,6 +11,7 @@ Exhaustive over the B200 axes (north star (4)):
             (paper: partially unrolled top-looking, n_b = NB)
       PANEL/PTMEM/RTMA/RTMAP  see include/bspotrf.h
       QTM   P threads per matrix (4, 8), TMEM columns per CTA (256, 512), n > 32
+      RCW   8 warps per 32 matrices, CTAs per SM (1, 2), n > 32
   * threads per block       -- 32..256
 Each point: regenerate the batch in place (device generator), flush L2, time
 ONE launch with CUDA events; median of --reps.  Every point is also checked
@@ -100,6 +101,8 @@ def candidates(n, chunk):
             if gen_instances.qtm_fits(n, p_, cols, pre):
                 c.append(dict(variant=bsp.VARIANT_QTM, threads_per_block=128, param=p_,
                               staging=gen_instances.qtm_staging(cols, pre)))
+        for k in gen_instances.rcw_ncta(n):
+            c.append(dict(variant=bsp.VARIANT_RCW, threads_per_block=256, param=k, staging=0))
     for nb in (2, 4, 8):
         if nb <= n or nb == 2:
             for tpb in (64, 128, 256):
@@ -117,7 +120,7 @@ def main():
     ap.add_argument("--kind", default="dd")
     ap.add_argument("--skip-from", action="append", default=[],
                     help="JSONL files whose points are already measured")
-    ap.add_argument("--variants", default="1,2,3,4,5,6,7,8")   # 9 (REGX) on request
+    ap.add_argument("--variants", default="1,2,3,4,5,6,7,8,10")   # 9 (REGX) on request
     a = ap.parse_args()
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     done = set()

@@ -49,6 +49,16 @@ def regx_combos(n):
 QTM_N = range(33, 65)
 QTM_COMBOS = ((4, 512, False), (4, 256, False), (4, 256, True), (4, 512, True), (8, 256, False))
 QTM_CT = (32, 0)
+RCW_N = range(33, 65)
+RCW_CT = (32, 0)
+
+
+def rcw_ncta(n):
+    """CTAs per SM of variant RCW: 2 (256 TMEM columns each) needs 4R(R-1) <= 128."""
+    r = (n + 7) // 8
+    return (1, 2) if 4 * r * (r - 1) <= 128 else (1,)
+
+
 TILE_N = range(1, 65)
 TILE_NB = (2, 4, 8)
 POTRS_N = range(1, 65)
@@ -230,6 +240,16 @@ def main():
                                f"&launch_qtm<{n}, {ct}, {p}, {cols}, {pr}>}}")
         body.append("}  // namespace bsp\n")
         name = f"inst_qtm_{n:02d}.cu"
+        write_if_changed(os.path.join(GEN, name), "\n".join(body))
+        files.add(name)
+    for n in RCW_N:
+        body = [hdr, '#include "../potrf_rcw.cuh"', "namespace bsp {"]
+        for k in rcw_ncta(n):
+            for ct in RCW_CT:
+                body.append(f"template cudaError_t launch_rcw<{n}, {ct}, {k}>(const FactorArgs &);")
+                entries.append(f"{{10, {n}, {k}, {ct}, 0, &launch_rcw<{n}, {ct}, {k}>}}")
+        body.append("}  // namespace bsp\n")
+        name = f"inst_rcw_{n:02d}.cu"
         write_if_changed(os.path.join(GEN, name), "\n".join(body))
         files.add(name)
     for n in TILE_N:

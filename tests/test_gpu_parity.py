@@ -106,6 +106,46 @@ def test_qtm_parity_failures_ragged(n, chunk):
         assert_parity(n, batch, chunk, canon, inter, out, info, cnt)
 
 
+def _rcw_ncta(n):
+    g = gen_instances_mod()
+    return g.rcw_ncta(n) if n in g.RCW_N else ()
+
+
+@pytest.mark.parametrize("n", [33, 34, 39, 40, 41, 47, 48, 49, 55, 56, 57, 61, 63, 64])
+@pytest.mark.parametrize("chunk", [32, 0, 96])
+def test_rcw_parity_failures_ragged(n, chunk):
+    """Variant RCW (8 warps share 32 matrices, factor in TMEM): every CTAs-per-SM
+    instance against the oracle and bitwise against the Fig. 9 emulator, with
+    injected failures, a batch that is not a multiple of 32, every n mod 8, and
+    the runtime-stride path (chunk 0, 96)."""
+    batch = 5 * 32 + 13
+    canon, inter = make_batch(n, batch, chunk, kind="dd", seed=n + 11, fail_seed=2018, fail_period=5)
+    failed, kk = synth.fail_plan(n, 2018, 5, np.arange(batch, dtype=np.uint64))
+    assert _rcw_ncta(n)
+    for k in _rcw_ncta(n):
+        t = dict(variant=bsp.VARIANT_RCW, threads_per_block=256, param=k, staging=0)
+        out, info, cnt = run_gpu(n, batch, chunk, inter, tune=t)
+        assert np.array_equal(info, np.where(failed, kk + 1, 0)), t
+        assert_parity(n, batch, chunk, canon, inter, out, info, cnt)
+
+
+@pytest.mark.parametrize("n", [36, 48, 52, 64])
+def test_rcw_integer_and_als(n):
+    """RCW on the exactness set (P2: returns exactly L0) and on ALS-shaped input."""
+    batch = 2 * 32 + 5
+    for k in _rcw_ncta(n):
+        t = dict(variant=bsp.VARIANT_RCW, threads_per_block=256, param=k, staging=0)
+        canon, inter = make_batch(n, batch, 32, kind="l0", seed=9)
+        out, info, _ = run_gpu(n, batch, 32, inter, tune=t)
+        assert (info == 0).all()
+        got = layout.from_interleaved(n, batch, 32, out).reshape(-1, n, n).transpose(0, 2, 1)
+        L0 = synth.l0_factor(n, 9, np.arange(batch, dtype=np.uint64))
+        assert np.array_equal(np.tril(got).astype(np.float64), L0)
+        canon, inter = make_batch(n, batch, 32, kind="als", seed=4)
+        out, info, cnt = run_gpu(n, batch, 32, inter, tune=t)
+        assert_parity(n, batch, 32, canon, inter, out, info, cnt)
+
+
 @pytest.mark.parametrize("n", [1, 2, 3, 5, 8, 11, 12, 16])
 @pytest.mark.parametrize("chunk", [32, 0, 96])
 def test_regx_multi_matrix_and_fast_math(n, chunk):
@@ -150,6 +190,8 @@ def _tunings(n, chunk):
     for p_, cols, pre in _qtm_combos(n):
         out.append(dict(variant=bsp.VARIANT_QTM, threads_per_block=128, param=p_,
                         staging=gen_instances_mod().qtm_staging(cols, pre)))
+    for k in _rcw_ncta(n):
+        out.append(dict(variant=bsp.VARIANT_RCW, threads_per_block=256, param=k, staging=0))
     for tpb in (64, 256):
         for nb in (2, 4, 8):
             if nb <= n or nb == 2:
