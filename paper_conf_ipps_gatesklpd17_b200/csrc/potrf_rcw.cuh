@@ -19,12 +19,18 @@
 //     "b" operand every warp needs) are published to a row buffer RB(c) in
 //     shared memory by their owners while those owners stream them out of TMEM
 //     for their own GEMM in block c-1 (no extra TMEM reads);
-//   * the input streams in one block ahead (cp.async, each thread copies the
-//     elements it will read itself, so only its own completion is awaited).
-//     Shared memory is two halves of R units of 8 KB; in block c the half
-//     c % 2 holds RB(c) in units 0..c-1 and the input stage of block c in
-//     units c..R-1, the other half receives RB(c+1) and stage(c+1): exactly
-//     16 units at any time (RB grows as the stage shrinks).
+//   * the input streams in one block ahead.  Shared memory is two halves of R
+//     units of 8 KB; block t (counted over all groups a persistent CTA
+//     processes) uses half t % 2: RB(c) in units 0..c-1 and the input stage of
+//     block c in units c..R-1, while the other half receives RB(c+1) and
+//     stage(c+1) -- 16 units at any time (RB grows as the stage shrinks).  The
+//     stage is column-run ordered, [w][i - 8c][lane], so for chunk 32 (one
+//     chunk = one group) each column j of the block is ONE contiguous run of
+//     (n - j) * 128 B: one TMA bulk copy per column (one mbarrier per half);
+//     other chunks use per-thread cp.async; results go out as coalesced
+//     per-thread streaming stores (one 128-B line per warp instruction);
+//   * persistent CTAs: the last block of a group prefetches block 0 of the
+//     CTA's next group, so loads never drain between groups.
 // Op order per element (i, j): fma with k = 0, 1, ..., j-1 ascending (GEMM over
 // k < 8c, then the in-block triangular updates), then mul by rcp.rn(L_jj) --
 // the Fig. 9 sequence of every other variant, so the output is bitwise
@@ -53,6 +59,13 @@ struct RcwShape {
     static constexpr int UNIT = W * W * 32;              // floats per 8 KB unit
     __host__ __device__ static constexpr int off(int r) { return 4 * r * (r - 1); }
     __host__ __device__ static constexpr int dt(int m, int k) { return m * (m + 1) / 2 + k; }
+    __host__ __device__ static constexpr int rs(int c) { return N - W * c; }   // stage row stride
+    __host__ __device__ static constexpr uint32_t bytes(int c) {                // TMA bytes of block c
+        uint32_t b = 0;
+        for (int w = 0; w < W; ++w)
+            if (W * c + w < N) b += (uint32_t)(N - W * c - w) * 128u;
+        return b;
+    }
     static constexpr size_t SMEM = (size_t)(2 * R * UNIT + 36 * 32) * sizeof(float);
     static_assert(off(R) <= HALF, "slots exceed the TMEM column budget");
 };
@@ -63,13 +76,13 @@ potrf_rcw_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__r
                  int64_t batch, int64_t cs) {
     using SH = RcwShape<N, NCTA>;
     constexpr int R = SH::R, UNIT = SH::UNIT;
+    constexpr bool TMA = CT == 32;                       // one chunk == one group of 32
     extern __shared__ __align__(16) float smf[];
     __shared__ uint32_t tmem_base_sh;
+    __shared__ __align__(8) uint64_t mbar[2];
 
     const int h = threadIdx.x >> 5, q = threadIdx.x & 31;
-    const int64_t gm = (int64_t)blockIdx.x * 32 + q;
-    const bool active = gm < batch;
-    const Addr<N, CT> ad(A, active ? gm : batch - 1, cs);
+    const int64_t ngroups = (batch + 31) / 32;
     float *DB = smf + 2 * R * UNIT;                      // diagonal block gather [36][32]
     auto unit = [&](int half, int u) { return smf + (size_t)(half * R + u) * UNIT; };
 
@@ -77,139 +90,176 @@ potrf_rcw_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__r
         tmem_alloc(&tmem_base_sh, SH::COLS);
         tmem_relinquish();
     }
+    if (TMA && threadIdx.x == 0) {
+        mbar_init(&mbar[0], 1);
+        mbar_init(&mbar[1], 1);
+        mbar_fence_init();
+    }
     tmem_fence_before();
     __syncthreads();
     tmem_fence_after();
     const uint32_t tb = tmem_base_sh + ((uint32_t)(32 * (h & 3)) << 16) + (uint32_t)((h >> 2) * SH::HALF);
 
-    // input of column block c -> stage units c..R-1 of half c % 2: element
-    // (8r+h, 8c+w) at [w][h][q] of unit r; only my own rows, lower part only
-    auto prefetch = [&](auto c_) {
+    // input of column block c of group g -> stage units c..R-1 of `half`:
+    // element (i, 8c+w) at [w][i - 8c][q]; lower part only
+    auto prefetch = [&](auto c_, int64_t g, int half) {
         constexpr int c = BSP_CI(c_);
-        sfor<c, R>([&](auto r_) {
-            constexpr int r = BSP_CI(r_);
-            const int i = 8 * r + h;
-            if (i < N) {
-                float *dst = unit(c & 1, r) + h * 32 + q;
-#pragma unroll
-                for (int w = 0; w < 8; ++w)
-                    if (8 * c + w < N && (r > c || w <= h)) cp_async4(dst + w * 256, ad.at(i, 8 * c + w));
-            }
-        });
-        cp_async_commit();
-    };
-    prefetch(std::integral_constant<int, 0>{});
-
-    int inf = 0;
-    float acc[R][8];
-    sfor<0, R>([&](auto c_) {
-        constexpr int c = BSP_CI(c_);
-        cp_async_wait<0>();                              // my stage(c) copies landed
-        __syncthreads();                                 // RB(c) published; old units free
-        if constexpr (c + 1 < R) prefetch(std::integral_constant<int, c + 1>{});
-
-        // (a) accumulators of my live rows = A(8r+h, 8c..8c+7)
-        sfor<c, R>([&](auto r_) {
-            constexpr int r = BSP_CI(r_);
-            const float *src = unit(c & 1, r) + h * 32 + q;
-#pragma unroll
-            for (int w = 0; w < 8; ++w)
-                acc[r][w] = (r > c || w <= h) && 8 * c + w < N ? src[w * 256] : 0.0f;
-        });
-
-        // (b) acc(r) -= L(8r+h, 0..8c-1) L(8c..8c+7, 0..8c-1)^T, k ascending; the
-        //     rows of block c+1 (my slot c+1) are published to RB(c+1) on the way
-        if constexpr (c > 0) {
-            const float4 *rb = reinterpret_cast<const float4 *>(unit(c & 1, 0)) + q;
-            float4 *rbn = reinterpret_cast<float4 *>(unit((c + 1) & 1, 0)) + h * 32 + q;
-#pragma unroll 1
-            for (int kq = 0; kq < 2 * c; ++kq) {
-                float b[8][4];
+        float *stg = unit(half, c);
+        if constexpr (TMA) {
+            if (threadIdx.x == 0) {
+                const float *chunk = A + g * (int64_t)(32 * N * N);
+                mbar_arrive_expect_tx(&mbar[half], SH::bytes(c));
 #pragma unroll
                 for (int w = 0; w < 8; ++w) {
-                    const float4 x = rb[(kq * 8 + w) * 32];
-                    b[w][0] = x.x, b[w][1] = x.y, b[w][2] = x.z, b[w][3] = x.w;
+                    const int j = 8 * c + w;
+                    if (j < N)
+                        bulk_g2s(stg + (w * SH::rs(c) + w) * 32, chunk + (j + j * N) * 32,
+                                 (uint32_t)((N - j) * 128), &mbar[half]);
                 }
-                float a[R][4];
-                sfor<c, R>([&](auto r_) {
-                    constexpr int r = BSP_CI(r_);
-                    tmem_ld4(tb + (uint32_t)(SH::off(r) + 4 * kq), a[r]);
-                });
-                tmem_wait_ld();
-                if constexpr (c + 1 < R) rbn[kq * 256] = make_float4(a[c + 1][0], a[c + 1][1], a[c + 1][2], a[c + 1][3]);
-                sfor<c, R>([&](auto r_) {
-                    constexpr int r = BSP_CI(r_);
-#pragma unroll
-                    for (int kk = 0; kk < 4; ++kk)
-#pragma unroll
-                        for (int w = 0; w < 8; ++w) acc[r][w] = f_upd(acc[r][w], a[r][kk], b[w][kk]);
-                });
             }
+        } else {
+            const int64_t gm = g * 32 + q;
+            const Addr<N, CT> ad(A, gm < batch ? gm : batch - 1, cs);
+            sfor<c, R>([&](auto r_) {
+                constexpr int r = BSP_CI(r_);
+                const int i = 8 * r + h;
+                if (i < N) {
+#pragma unroll
+                    for (int w = 0; w < 8; ++w)
+                        if (8 * c + w < N && (r > c || w <= h))
+                            cp_async4(stg + (w * SH::rs(c) + i - 8 * c) * 32 + q, ad.at(i, 8 * c + w));
+                }
+            });
+            cp_async_commit();
         }
+    };
+    int64_t g = blockIdx.x;
+    int ph = 0;                                          // half of the group's block 0
+    uint32_t par = 0;                                    // mbarrier phase bits, one per half
+    if (g < ngroups) prefetch(std::integral_constant<int, 0>{}, g, ph);
 
-        // (c) diagonal block: gather rows 8c..8c+7, factor it in every warp (identical bits)
-#pragma unroll
-        for (int m = 0; m < 8; ++m)
-            if (m == h && 8 * c + m < N) {
-#pragma unroll
-                for (int w = 0; w <= m; ++w) DB[SH::dt(m, w) * 32 + q] = acc[c][w];
+    float acc[R][8];
+    for (; g < ngroups; g += gridDim.x) {
+        const int64_t gm = g * 32 + q;
+        const bool active = gm < batch;
+        const Addr<N, CT> ad(A, active ? gm : batch - 1, cs);
+        int inf = 0;
+        sfor<0, R>([&](auto c_) {
+            constexpr int c = BSP_CI(c_);
+            const int half = (c + ph) & 1;
+            if constexpr (TMA) {
+                mbar_wait(&mbar[half], (par >> half) & 1);
+                par ^= 1u << half;
+            } else {
+                cp_async_wait<0>();                      // my stage(c) copies landed
             }
-        __syncthreads();
-        float d[36], inv[8];
+            __syncthreads();                             // RB(c) published; old units free
+            if constexpr (c + 1 < R) prefetch(std::integral_constant<int, c + 1>{}, g, half ^ 1);
+            else if (g + gridDim.x < ngroups) prefetch(std::integral_constant<int, 0>{}, g + gridDim.x, half ^ 1);
+            const float *stg = unit(half, c) + q;
+
+            // (a) accumulators of my live rows = A(8r+h, 8c..8c+7)
+            sfor<c, R>([&](auto r_) {
+                constexpr int r = BSP_CI(r_);
+                const float *src = stg + (8 * (r - c) + h) * 32;
 #pragma unroll
-        for (int t = 0; t < 36; ++t) d[t] = DB[t * 32 + q];
+                for (int w = 0; w < 8; ++w)
+                    acc[r][w] = (r > c || w <= h) && 8 * c + w < N ? src[w * SH::rs(c) * 32] : 0.0f;
+            });
+
+            // (b) acc(r) -= L(8r+h, 0..8c-1) L(8c..8c+7, 0..8c-1)^T, k ascending; the
+            //     rows of block c+1 (my slot c+1) are published to RB(c+1) on the way
+            if constexpr (c > 0) {
+                const float4 *rb = reinterpret_cast<const float4 *>(unit(half, 0)) + q;
+                float4 *rbn = reinterpret_cast<float4 *>(unit(half ^ 1, 0)) + h * 32 + q;
+#pragma unroll 1
+                for (int kq = 0; kq < 2 * c; ++kq) {
+                    float b[8][4];
 #pragma unroll
-        for (int k = 0; k < 8; ++k) {
-            if (8 * c + k >= N) break;
-            const float p = d[SH::dt(k, k)];
-            pivot_check(p, 8 * c + k, inf);
-            const float s = f_sqrt(p);
-            d[SH::dt(k, k)] = s;
-            inv[k] = f_rcp(s);
+                    for (int w = 0; w < 8; ++w) {
+                        const float4 x = rb[(kq * 8 + w) * 32];
+                        b[w][0] = x.x, b[w][1] = x.y, b[w][2] = x.z, b[w][3] = x.w;
+                    }
+                    float a[R][4];
+                    sfor<c, R>([&](auto r_) {
+                        constexpr int r = BSP_CI(r_);
+                        tmem_ld4(tb + (uint32_t)(SH::off(r) + 4 * kq), a[r]);
+                    });
+                    tmem_wait_ld();
+                    if constexpr (c + 1 < R) rbn[kq * 256] = make_float4(a[c + 1][0], a[c + 1][1], a[c + 1][2], a[c + 1][3]);
+                    sfor<c, R>([&](auto r_) {
+                        constexpr int r = BSP_CI(r_);
 #pragma unroll
-            for (int m = k + 1; m < 8; ++m) d[SH::dt(m, k)] = f_mul(d[SH::dt(m, k)], inv[k]);
+                        for (int kk = 0; kk < 4; ++kk)
 #pragma unroll
-            for (int j = k + 1; j < 8; ++j)
-#pragma unroll
-                for (int m = j; m < 8; ++m) d[SH::dt(m, j)] = f_upd(d[SH::dt(m, j)], d[SH::dt(m, k)], d[SH::dt(j, k)]);
-        }
-        if (active) {
+                            for (int w = 0; w < 8; ++w) acc[r][w] = f_upd(acc[r][w], a[r][kk], b[w][kk]);
+                    });
+                }
+            }
+
+            // (c) diagonal block: gather rows 8c..8c+7, factor it in every warp (identical bits)
 #pragma unroll
             for (int m = 0; m < 8; ++m)
                 if (m == h && 8 * c + m < N) {
 #pragma unroll
-                    for (int w = 0; w <= m; ++w) st_stream(ad.at(8 * c + m, 8 * c + w), d[SH::dt(m, w)]);
+                    for (int w = 0; w <= m; ++w) DB[SH::dt(m, w) * 32 + q] = acc[c][w];
                 }
-        }
-
-        // (d) triangular solve of my rows below the block; HBM, TMEM, RB(c+1)
-        sfor<c + 1, R>([&](auto r_) {
-            constexpr int r = BSP_CI(r_);
+            __syncthreads();
+            float d[36], inv[8];
+#pragma unroll
+            for (int t = 0; t < 36; ++t) d[t] = DB[t * 32 + q];
 #pragma unroll
             for (int k = 0; k < 8; ++k) {
                 if (8 * c + k >= N) break;
-                acc[r][k] = f_mul(acc[r][k], inv[k]);
+                const float p = d[SH::dt(k, k)];
+                pivot_check(p, 8 * c + k, inf);
+                const float s = f_sqrt(p);
+                d[SH::dt(k, k)] = s;
+                inv[k] = f_rcp(s);
 #pragma unroll
-                for (int j = k + 1; j < 8; ++j) acc[r][j] = f_upd(acc[r][j], acc[r][k], d[SH::dt(j, k)]);
-            }
-            const int i = 8 * r + h;
-            if (active && i < N) {
+                for (int m = k + 1; m < 8; ++m) d[SH::dt(m, k)] = f_mul(d[SH::dt(m, k)], inv[k]);
 #pragma unroll
-                for (int w = 0; w < 8; ++w)
-                    if (8 * c + w < N) st_stream(ad.at(i, 8 * c + w), acc[r][w]);
+                for (int j = k + 1; j < 8; ++j)
+#pragma unroll
+                    for (int m = j; m < 8; ++m) d[SH::dt(m, j)] = f_upd(d[SH::dt(m, j)], d[SH::dt(m, k)], d[SH::dt(j, k)]);
             }
-            tmem_st8(tb + (uint32_t)(SH::off(r) + 8 * c), acc[r]);
-            if constexpr (r == c + 1) {
-                float4 *rbn = reinterpret_cast<float4 *>(unit((c + 1) & 1, 0)) + h * 32 + q;
-                rbn[(2 * c) * 256] = make_float4(acc[r][0], acc[r][1], acc[r][2], acc[r][3]);
-                rbn[(2 * c + 1) * 256] = make_float4(acc[r][4], acc[r][5], acc[r][6], acc[r][7]);
-            }
-        });
-        tmem_wait_st();
-    });
+#pragma unroll
+            for (int m = 0; m < 8; ++m)
+                if (m == h && 8 * c + m < N) {
+#pragma unroll
+                    for (int w = 0; w <= m; ++w)
+                        if (active) st_stream(ad.at(8 * c + m, 8 * c + w), d[SH::dt(m, w)]);
+                }
 
-    if (active && h == 0) info[gm] = inf;
-    if (h == 0) count_failures(active && inf != 0, nfailed);
+            // (d) triangular solve of my rows below the block; out, TMEM, RB(c+1)
+            sfor<c + 1, R>([&](auto r_) {
+                constexpr int r = BSP_CI(r_);
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    if (8 * c + k >= N) break;
+                    acc[r][k] = f_mul(acc[r][k], inv[k]);
+#pragma unroll
+                    for (int j = k + 1; j < 8; ++j) acc[r][j] = f_upd(acc[r][j], acc[r][k], d[SH::dt(j, k)]);
+                }
+                const int i = 8 * r + h;
+                if (active && i < N) {
+#pragma unroll
+                    for (int w = 0; w < 8; ++w)
+                        if (8 * c + w < N) st_stream(ad.at(i, 8 * c + w), acc[r][w]);
+                }
+                tmem_st8(tb + (uint32_t)(SH::off(r) + 8 * c), acc[r]);
+                if constexpr (r == c + 1) {
+                    float4 *rbn = reinterpret_cast<float4 *>(unit(half ^ 1, 0)) + h * 32 + q;
+                    rbn[(2 * c) * 256] = make_float4(acc[r][0], acc[r][1], acc[r][2], acc[r][3]);
+                    rbn[(2 * c + 1) * 256] = make_float4(acc[r][4], acc[r][5], acc[r][6], acc[r][7]);
+                }
+            });
+            tmem_wait_st();
+        });
+        if (active && h == 0) info[gm] = inf;
+        if (h == 0) count_failures(active && inf != 0, nfailed);
+        ph = (ph + R) & 1;
+    }
 
     tmem_fence_before();
     __syncthreads();
@@ -228,9 +278,18 @@ cudaError_t launch_rcw(const FactorArgs &a) {
     size_t sm = SH::SMEM;
     if constexpr (NCTA == 1)
         if (sm < (size_t)116 * 1024) sm = (size_t)116 * 1024;
-    const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
-    kern<<<grid_for(a.batch, 32), 256, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
+    static int nsm = 0;                                  // persistent grid: NCTA CTAs per SM
+    if (nsm == 0) {
+        int dev = 0;
+        e = cudaGetDevice(&dev);
+        if (e == cudaSuccess) e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+        if (e != cudaSuccess) return e;
+    }
+    const int64_t groups = (a.batch + 31) / 32;
+    const int64_t grid = groups < (int64_t)nsm * NCTA ? groups : (int64_t)nsm * NCTA;
+    kern<<<(unsigned)grid, 256, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
     return cudaGetLastError();
 }
 
