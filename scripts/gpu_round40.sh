@@ -5,5 +5,5 @@ mkdir -p gpurun_out
 python -c "import oracle; oracle.build()" > /dev/null 2>&1
 timeout 600 python -m pytest tests/test_gpu_parity.py -q -x -p no:cacheprovider -k "rcw or bitwise" > gpurun_out/pytest_rcw.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_rcw.log
 tail -n 3 gpurun_out/pytest_rcw.log
-timeout 1200 python scripts/autotune.py --n 33-64 --chunks 32,0 --variants 10 --reps 3 --out gpurun_out/sweep_rcw6.jsonl > gpurun_out/sweep_rcw6.log 2>&1
-tail -n 1 gpurun_out/sweep_rcw6.log
+timeout 1200 python scripts/autotune.py --n 33-64 --chunks 32,0 --variants 10 --reps 3 --out gpurun_out/sweep_rcw7.jsonl > gpurun_out/sweep_rcw7.log 2>&1
+tail -n 1 gpurun_out/sweep_rcw7.log
