@@ -85,12 +85,17 @@ enum {
                                  tolerance-checked, not bitwise reproducible,
                                  never chosen by the default table), 0 = IEEE;
                                  <= 128 threads per block; 1 <= n <= 16       */
-    BSPOTRF_VARIANT_RCW = 10  /* row-cyclic warps: 8 warps share 32 matrices
+    BSPOTRF_VARIANT_RCW = 10, /* row-cyclic warps: 8 warps share 32 matrices
                                  (lane = matrix), warp h owns rows 8r+h, the
                                  factor in Tensor Memory, left-looking over
                                  8-wide column blocks; `param` = CTAs per SM
                                  (1: 512 TMEM columns, any n; 2: 256 each,
                                  n <= 48); any chunk; 33 <= n <= 64           */
+    BSPOTRF_VARIANT_REGV = 11 /* REG with 128-bit accesses: each thread owns 4
+                                 adjacent matrices (one float4 per element);
+                                 needs C % 4 == 0 (C = chunk, or batch when
+                                 chunk == 0), else runs REG (same bits);
+                                 <= 128 threads per block; 1 <= n <= 8        */
 };
 
 /* Launch tuning (a row of the autotuning table). */

@@ -66,6 +66,11 @@ cudaError_t launch_qtm(const FactorArgs &a);
 template <int N, int CT, int NCTA>
 cudaError_t launch_rcw(const FactorArgs &a);
 
+// Variant REGV: REG with four adjacent matrices per thread and 128-bit
+// accesses (csrc/potrf_regv.cuh); falls back to REG when C % 4 != 0.
+template <int N>
+cudaError_t launch_regv(const FactorArgs &a);
+
 // Variant TILE: the paper's top-looking tile algorithm, NB x NB register
 // tiles streamed from global memory, runtime chunk stride (csrc/potrf_tile.cuh).
 template <int N, int NB>

@@ -12,6 +12,7 @@ Exhaustive over the B200 axes (north star (4)):
       PANEL/PTMEM/RTMA/RTMAP  see include/bspotrf.h
       QTM   P threads per matrix (4, 8), TMEM columns per CTA (256, 512), n > 32
       RCW   8 warps per 32 matrices, CTAs per SM (1, 2), n > 32
+      REGV  4 adjacent matrices per thread, 128-bit accesses, n <= 8
   * threads per block       -- 32..256
 Each point: regenerate the batch in place (device generator), flush L2, time
 ONE launch with CUDA events; median of --reps.  Every point is also checked
@@ -94,6 +95,9 @@ def candidates(n, chunk):
         for m, fast in gen_instances.regx_combos(n):
             for tpb in (64, 128):
                 c.append(dict(variant=bsp.VARIANT_REGX, threads_per_block=tpb, param=m, staging=int(fast)))
+    if n <= 8:
+        for tpb in (64, 128):
+            c.append(dict(variant=bsp.VARIANT_REGV, threads_per_block=tpb, param=0, staging=0))
     if 33 <= n <= 64:
         sys.path.insert(0, os.path.join(ROOT, "scripts"))
         import gen_instances
@@ -120,7 +124,7 @@ def main():
     ap.add_argument("--kind", default="dd")
     ap.add_argument("--skip-from", action="append", default=[],
                     help="JSONL files whose points are already measured")
-    ap.add_argument("--variants", default="1,2,3,4,5,6,7,8,10")   # 9 (REGX) on request
+    ap.add_argument("--variants", default="1,2,3,4,5,6,7,8,10,11")   # 9 (REGX) on request
     a = ap.parse_args()
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     done = set()

@@ -49,6 +49,7 @@ def regx_combos(n):
 QTM_N = range(33, 65)
 QTM_COMBOS = ((4, 512, False), (4, 256, False), (4, 256, True), (4, 512, True), (8, 256, False))
 QTM_CT = (32, 0)
+REGV_N = range(1, 9)
 RCW_N = range(33, 65)
 RCW_CT = (32, 0)
 
@@ -240,6 +241,14 @@ def main():
                                f"&launch_qtm<{n}, {ct}, {p}, {cols}, {pr}>}}")
         body.append("}  // namespace bsp\n")
         name = f"inst_qtm_{n:02d}.cu"
+        write_if_changed(os.path.join(GEN, name), "\n".join(body))
+        files.add(name)
+    for n in REGV_N:
+        body = [hdr, '#include "../potrf_regv.cuh"', "namespace bsp {"]
+        body.append(f"template cudaError_t launch_regv<{n}>(const FactorArgs &);")
+        entries.append(f"{{11, {n}, 0, 0, 0, &launch_regv<{n}>}}")
+        body.append("}  // namespace bsp\n")
+        name = f"inst_regv_{n:02d}.cu"
         write_if_changed(os.path.join(GEN, name), "\n".join(body))
         files.add(name)
     for n in RCW_N:

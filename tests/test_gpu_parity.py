@@ -146,6 +146,22 @@ def test_rcw_integer_and_als(n):
         assert_parity(n, batch, 32, canon, inter, out, info, cnt)
 
 
+@pytest.mark.parametrize("n", [1, 2, 3, 4, 5, 6, 7, 8])
+@pytest.mark.parametrize("chunk,batch", [(32, 3 * 512 + 37), (0, 4 * 301), (0, 4 * 301 + 1), (96, 999), (64, 2)])
+def test_regv_128bit_groups(n, chunk, batch):
+    """Variant REGV (4 adjacent matrices per thread, float4 accesses): bitwise equal to
+    the Fig. 9 emulator and O1-O4 (pad lanes untouched when a group straddles the end
+    of the batch), with injected failures; chunk 0 with batch % 4 != 0 takes the REG
+    fallback."""
+    canon, inter = make_batch(n, batch, chunk, kind="dd", seed=n + 21, fail_seed=2018, fail_period=6)
+    failed, kk = synth.fail_plan(n, 2018, 6, np.arange(batch, dtype=np.uint64))
+    for tpb in (64, 128):
+        t = dict(variant=bsp.VARIANT_REGV, threads_per_block=tpb, param=0, staging=0)
+        out, info, cnt = run_gpu(n, batch, chunk, inter, tune=t)
+        assert np.array_equal(info, np.where(failed, kk + 1, 0)), t
+        assert_parity(n, batch, chunk, canon, inter, out, info, cnt)
+
+
 @pytest.mark.parametrize("n", [1, 2, 3, 5, 8, 11, 12, 16])
 @pytest.mark.parametrize("chunk", [32, 0, 96])
 def test_regx_multi_matrix_and_fast_math(n, chunk):
@@ -192,6 +208,8 @@ def _tunings(n, chunk):
                         staging=gen_instances_mod().qtm_staging(cols, pre)))
     for k in _rcw_ncta(n):
         out.append(dict(variant=bsp.VARIANT_RCW, threads_per_block=256, param=k, staging=0))
+    if n <= 8:
+        out.append(dict(variant=bsp.VARIANT_REGV, threads_per_block=128, param=0, staging=0))
     for tpb in (64, 256):
         for nb in (2, 4, 8):
             if nb <= n or nb == 2:
