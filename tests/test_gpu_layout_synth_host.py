@@ -73,7 +73,7 @@ def test_generator_partition_invariance_chunk0():
 
 @pytest.mark.parametrize("n,chunk,slab", [(8, 32, 0), (16, 32, 4096), (16, 64, 3 * 64),
                                           (21, 32, 1024), (32, 32, 2048), (5, 0, 500), (40, 0, 0),
-                                          (12, 128, 256)])
+                                          (12, 128, 256), (48, 32, 1024), (64, 64, 640)])
 def test_host_end_to_end(n, chunk, slab):
     torch = torch_mod()
     batch = 5000 + 13
