@@ -105,6 +105,9 @@ def candidates(n, chunk):
             if gen_instances.qtm_fits(n, p_, cols, pre):
                 c.append(dict(variant=bsp.VARIANT_QTM, threads_per_block=128, param=p_,
                               staging=gen_instances.qtm_staging(cols, pre)))
+    sys.path.insert(0, os.path.join(ROOT, "scripts"))
+    import gen_instances
+    if n in gen_instances.RCW_N:
         for k in gen_instances.rcw_ncta(n):
             c.append(dict(variant=bsp.VARIANT_RCW, threads_per_block=256, param=k, staging=0))
     for nb in (2, 4, 8):
