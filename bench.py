@@ -262,6 +262,18 @@ class ClockSampler:
         if self._win:
             self._win[-1][1] = time.perf_counter()
 
+    def sample_now(self, k=3):
+        """Synchronous samples from the calling thread while queued kernels run
+        (short timed regions can end before the sampler thread gets a turn)."""
+        if self.nv is None:
+            return
+        for _ in range(k):
+            try:
+                self._all.append((time.perf_counter(), self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM),
+                                  int(self._rfn(self.h))))
+            except Exception:
+                pass
+
     def stop(self):
         if self._t is not None:
             self._stop.set()
@@ -371,6 +383,7 @@ def run_ours(a, w):
                 dist.all_reduce(pool[i][2])
             ev[i][1].record(stream)
         e1.record(stream)
+        clk.sample_now()                       # the queued steps are running now
         torch.cuda.synchronize(dev)
         clk.mark_stop()
         barrier()
