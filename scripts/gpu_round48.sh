@@ -1,0 +1,9 @@
+#!/bin/bash
+# RCW + output staging with bulk stores (one CTA/SM, R <= 7): parity, sweep n = 33..64 chunk 32.
+cd "$GRAFT_REPO_ROOT" || exit 1
+mkdir -p gpurun_out
+python -c "import oracle; oracle.build()" > /dev/null 2>&1
+timeout 600 python -m pytest tests/test_gpu_parity.py -q -x -p no:cacheprovider -k "rcw or bitwise" > gpurun_out/pytest_rcw.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_rcw.log
+tail -n 2 gpurun_out/pytest_rcw.log
+timeout 900 python scripts/autotune.py --n 33-64 --chunks 32 --variants 10 --reps 3 --out gpurun_out/sweep_rcw8.jsonl > gpurun_out/sweep_rcw8.log 2>&1
+tail -n 1 gpurun_out/sweep_rcw8.log
