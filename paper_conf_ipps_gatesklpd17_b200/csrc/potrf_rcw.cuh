@@ -280,13 +280,10 @@ cudaError_t launch_rcw(const FactorArgs &a) {
         if (sm < (size_t)116 * 1024) sm = (size_t)116 * 1024;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
-    static int nsm = 0;                                  // persistent grid: NCTA CTAs per SM
-    if (nsm == 0) {
-        int dev = 0;
-        e = cudaGetDevice(&dev);
-        if (e == cudaSuccess) e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-        if (e != cudaSuccess) return e;
-    }
+    int dev = 0, nsm = 0;                                // persistent grid: NCTA CTAs per SM
+    e = cudaGetDevice(&dev);                             // (queried per call: reentrant, any device)
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (e != cudaSuccess) return e;
     const int64_t groups = (a.batch + 31) / 32;
     const int64_t grid = groups < (int64_t)nsm * NCTA ? groups : (int64_t)nsm * NCTA;
     kern<<<(unsigned)grid, 256, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
