@@ -297,6 +297,7 @@ def run_ours(a, w):
     import torch.distributed as dist
 
     import paper_conf_ipps_gatesklpd17_b200 as bsp
+    from paper_conf_ipps_gatesklpd17_b200 import multi_gpu
 
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -310,7 +311,6 @@ def run_ours(a, w):
     n, chunk, kind = w["n"], w["chunk"], w["kind"]
     fail_period = w.get("fail_period", 0)
     if w.get("global_batch"):                    # strong scaling: split one global batch
-        from paper_conf_ipps_gatesklpd17_b200 import multi_gpu
         b0, B = multi_gpu.rank_slice(w["batch"], world, rank, chunk)
     else:                                        # weak scaling: the batch is per GPU
         B = w["batch"]
@@ -392,12 +392,7 @@ def run_ours(a, w):
         launch_ms += steps_ms
         fails += sum(int(pool[i][2].item()) for i in range(g))   # global (all-reduced) counts
         done += g
-    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
-    lm = torch.tensor([statistics.mean(launch_ms)], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        dist.all_reduce(lm, op=dist.ReduceOp.MAX)
-    total_ms, mean_launch_ms = float(t.item()), float(lm.item())
+    total_ms, mean_launch_ms = multi_gpu.max_over_ranks([total_ms, statistics.mean(launch_ms)], device=dev)
     clk.stop()
     # correctness guard on the timed output: SPD input -> no failure; injected
     # failures -> the global count equals the enumerated plan (pin P10)
@@ -414,7 +409,8 @@ def run_ours(a, w):
 
     ms_per_step = total_ms / a.steps
     Btot = w["batch"] if w.get("global_batch") else world * B
-    value = Btot * flops_per_matrix(n) / (ms_per_step * 1e-3) / 1e9
+    value = multi_gpu.job_throughput(B, world, ms_per_step, flops_per_matrix(n),
+                                     global_units=w["batch"] if w.get("global_batch") else None)
     alg_bytes = B * bytes_per_matrix(n)
     achieved = alg_bytes / (mean_launch_ms * 1e-3) / 1e9
     peak, peak_src = measured_peak()

@@ -46,6 +46,25 @@ def allreduce_count(count, group=None):
     return int(count.item())
 
 
+def max_over_ranks(values, device=None, group=None):
+    """Device timings of a multi-GPU step: the MAX over ranks of each value
+    (the job is as slow as its slowest rank; bench.py's timing rule).  `values`
+    is a list of floats; returns the list of maxima (identity at world 1)."""
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([float(v) for v in values], dtype=torch.float64, device=device)
+    if dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX, group=group)
+    return [float(x) for x in t.tolist()]
+
+
+def job_throughput(units_per_rank, world, max_ms_per_step, flops_per_unit, global_units=None):
+    """Whole-job Gflop/s: every rank's units (or the global batch when the batch
+    is split) over the max-over-ranks step time."""
+    units = global_units if global_units is not None else units_per_rank * world
+    return units * flops_per_unit / (max_ms_per_step * 1e-3) / 1e9
+
+
 class RankBatch:
     """This rank's slice of a global synthetic batch, resident on its GPU."""
 

@@ -68,3 +68,35 @@ def test_gloo_allreduce_of_failure_count(world):
     assert all(r[4] == expected for r in res)
     assert sum(r[3] for r in res) == expected
     assert sum(r[2] for r in res) == B
+
+
+def _timing_worker(rank, world, port, q):
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK=str(rank),
+                      WORLD_SIZE=str(world), LOCAL_RANK=str(rank))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    # rank r "measured" a step time of 10 + 5r ms and a mean launch of 2 - r ms
+    total, launch = multi_gpu.max_over_ranks([10.0 + 5 * rank, 2.0 - rank])
+    value = multi_gpu.job_throughput(1 << 20, world, total, 16 ** 3 / 3)
+    q.put((rank, total, launch, value))
+    dist.destroy_process_group()
+
+
+def test_gloo_max_over_ranks_timing():
+    """bench.py's rule: the job's step time is the MAX over ranks (every rank
+    reports the same number) and the throughput is all ranks' units over it."""
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_timing_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted(q.get(timeout=120) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for _, total, launch, value in res:
+        assert total == 15.0 and launch == 2.0
+        assert abs(value - 2 * (1 << 20) * (16 ** 3 / 3) / 15e-3 / 1e9) < 1e-9
+    assert multi_gpu.max_over_ranks([3.5]) == [3.5]          # world 1: identity
