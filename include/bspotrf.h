@@ -91,11 +91,15 @@ enum {
                                  8-wide column blocks; `param` = CTAs per SM
                                  (1: 512 TMEM columns, any n; 2: 256 each,
                                  n <= 48); any chunk; 33 <= n <= 64           */
-    BSPOTRF_VARIANT_REGV = 11 /* REG with 128-bit accesses: each thread owns 4
+    BSPOTRF_VARIANT_REGV = 11, /* REG with 128-bit accesses: each thread owns 4
                                  adjacent matrices (one float4 per element);
                                  needs C % 4 == 0 (C = chunk, or batch when
                                  chunk == 0), else runs REG (same bits);
                                  <= 128 threads per block; 1 <= n <= 8        */
+    BSPOTRF_VARIANT_RCW16 = 12 /* RCW with 16 warps per 32 matrices (rows
+                                 16r+h), one CTA per SM; faster than RCW only
+                                 for the simple interleaved layout (chunk 0);
+                                 any chunk; 49 <= n <= 64                     */
 };
 
 /* Launch tuning (a row of the autotuning table). */

@@ -131,6 +131,11 @@ static LaunchFn resolve(int n, int chunk, const bspotrf_tuning &t, int *tpb_out)
         LaunchFn f = find(BSPOTRF_VARIANT_QTM, n, t.param, chunk == 32 ? 32 : 0, st);
         return f ? f : find(BSPOTRF_VARIANT_QTM, n, t.param, 0, st);
     }
+    case BSPOTRF_VARIANT_RCW16: {
+        *tpb_out = 512;
+        LaunchFn f = find(BSPOTRF_VARIANT_RCW16, n, 0, chunk == 32 ? 32 : 0, 0);
+        return f ? f : find(BSPOTRF_VARIANT_RCW16, n, 0, 0, 0);
+    }
     case BSPOTRF_VARIANT_REGV:
         return find(BSPOTRF_VARIANT_REGV, n, 0, 0, 0);
     case BSPOTRF_VARIANT_RCW: {

@@ -71,6 +71,11 @@ cudaError_t launch_rcw(const FactorArgs &a);
 template <int N>
 cudaError_t launch_regv(const FactorArgs &a);
 
+// Variant RCW16: RCW with 16 warps per 32 matrices (rows 16r+h), one CTA per SM
+// (csrc/potrf_rcw16.cuh).
+template <int N, int CT>
+cudaError_t launch_rcw16(const FactorArgs &a);
+
 // Variant TILE: the paper's top-looking tile algorithm, NB x NB register
 // tiles streamed from global memory, runtime chunk stride (csrc/potrf_tile.cuh).
 template <int N, int NB>

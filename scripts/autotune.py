@@ -110,6 +110,8 @@ def candidates(n, chunk):
     if n in gen_instances.RCW_N:
         for k in gen_instances.rcw_ncta(n):
             c.append(dict(variant=bsp.VARIANT_RCW, threads_per_block=256, param=k, staging=0))
+    if n in gen_instances.RCW16_N:
+        c.append(dict(variant=bsp.VARIANT_RCW16, threads_per_block=512, param=0, staging=0))
     for nb in (2, 4, 8):
         if nb <= n or nb == 2:
             for tpb in (64, 128, 256):
@@ -127,7 +129,7 @@ def main():
     ap.add_argument("--kind", default="dd")
     ap.add_argument("--skip-from", action="append", default=[],
                     help="JSONL files whose points are already measured")
-    ap.add_argument("--variants", default="1,2,3,4,5,6,7,8,10,11")   # 9 (REGX) on request
+    ap.add_argument("--variants", default="1,2,3,4,5,6,7,8,10,11,12")   # 9 (REGX) on request
     a = ap.parse_args()
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     done = set()

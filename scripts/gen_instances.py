@@ -51,6 +51,7 @@ QTM_COMBOS = ((4, 512, False), (4, 256, False), (4, 256, True), (4, 512, True), 
 QTM_CT = (32, 0)
 REGV_N = range(1, 9)
 RCW_N = range(33, 65)
+RCW16_N = range(49, 65)
 RCW_CT = (32, 0)
 
 
@@ -241,6 +242,15 @@ def main():
                                f"&launch_qtm<{n}, {ct}, {p}, {cols}, {pr}>}}")
         body.append("}  // namespace bsp\n")
         name = f"inst_qtm_{n:02d}.cu"
+        write_if_changed(os.path.join(GEN, name), "\n".join(body))
+        files.add(name)
+    for n in RCW16_N:
+        body = [hdr, '#include "../potrf_rcw16.cuh"', "namespace bsp {"]
+        for ct in RCW_CT:
+            body.append(f"template cudaError_t launch_rcw16<{n}, {ct}>(const FactorArgs &);")
+            entries.append(f"{{12, {n}, 0, {ct}, 0, &launch_rcw16<{n}, {ct}>}}")
+        body.append("}  // namespace bsp\n")
+        name = f"inst_rcw16_{n:02d}.cu"
         write_if_changed(os.path.join(GEN, name), "\n".join(body))
         files.add(name)
     for n in REGV_N:

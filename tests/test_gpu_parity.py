@@ -122,8 +122,10 @@ def test_rcw_parity_failures_ragged(n, chunk):
     canon, inter = make_batch(n, batch, chunk, kind="dd", seed=n + 11, fail_seed=2018, fail_period=5)
     failed, kk = synth.fail_plan(n, 2018, 5, np.arange(batch, dtype=np.uint64))
     assert _rcw_ncta(n)
-    for k in _rcw_ncta(n):
-        t = dict(variant=bsp.VARIANT_RCW, threads_per_block=256, param=k, staging=0)
+    ts = [dict(variant=bsp.VARIANT_RCW, threads_per_block=256, param=k, staging=0) for k in _rcw_ncta(n)]
+    if n in gen_instances_mod().RCW16_N:
+        ts.append(dict(variant=bsp.VARIANT_RCW16, threads_per_block=512, param=0, staging=0))
+    for t in ts:
         out, info, cnt = run_gpu(n, batch, chunk, inter, tune=t)
         assert np.array_equal(info, np.where(failed, kk + 1, 0)), t
         assert_parity(n, batch, chunk, canon, inter, out, info, cnt)
@@ -208,6 +210,8 @@ def _tunings(n, chunk):
                         staging=gen_instances_mod().qtm_staging(cols, pre)))
     for k in _rcw_ncta(n):
         out.append(dict(variant=bsp.VARIANT_RCW, threads_per_block=256, param=k, staging=0))
+    if n in gen_instances_mod().RCW16_N:
+        out.append(dict(variant=bsp.VARIANT_RCW16, threads_per_block=512, param=0, staging=0))
     if n <= 8:
         out.append(dict(variant=bsp.VARIANT_REGV, threads_per_block=128, param=0, staging=0))
     for tpb in (64, 256):
