@@ -383,7 +383,7 @@ def run_ours(a, w):
                 dist.all_reduce(pool[i][2])
             ev[i][1].record(stream)
         e1.record(stream)
-        clk.sample_now()                       # the queued steps are running now
+        clk.sample_now(1)                      # the queued steps are running now
         torch.cuda.synchronize(dev)
         clk.mark_stop()
         barrier()
