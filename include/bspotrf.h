@@ -97,8 +97,9 @@ enum {
                                  chunk == 0), else runs REG (same bits);
                                  <= 128 threads per block; 1 <= n <= 8        */
     BSPOTRF_VARIANT_RCW16 = 12 /* RCW with 16 warps per 32 matrices (rows
-                                 16r+h), one CTA per SM; faster than RCW only
-                                 for the simple interleaved layout (chunk 0);
+                                 16r+h), one CTA per SM; faster than RCW where
+                                 the input comes by per-thread copies (chunk
+                                 != 32), slower with chunk 32 (TMA path);
                                  any chunk; 49 <= n <= 64                     */
 };
 
