@@ -17,9 +17,25 @@ Contents
 * ``checks``           -- the acceptance metrics O1-O4.
 * ``metrics``          -- flop and byte models.
 
-Every function is pinned by ``tests/test_oracle_*.py`` against hand-worked
-values, closed forms, LAPACK, brute force or invariants; none is "parity
-unpinned".
+Pin map (what fixes each function other than itself; ``-m "not gpu"``):
+
+* ``potrf``             hand-worked 2x2/3x3/4x4 (golden/handworked_p1.json),
+                        integer L0 exactness, identity/diagonal, tridiagonal
+                        Toeplitz closed forms, info = k, LAPACK dpotrf
+                        (tests/test_oracle_pins.py)
+* ``potrs``             hand-worked systems (golden/handworked_solve_p11.json),
+                        integer systems, LAPACK dpotrs (tests/test_oracle_solve.py)
+* ``layout.offset`` / ``to_/from_interleaved``  Fig. 10 pointer walks replayed,
+                        hand-built layouts (tests/test_oracle_layout.py)
+* ``layout.rect_*``     hand-worked offsets and a value-naming scatter,
+                        square case == the matrix formula (test_oracle_layout.py)
+* ``checks.residual`` / ``solve_residual`` / ``strict_relative_error`` /
+  ``colnorm_error``     closed-form values of hand-perturbed 2x2/3x3 factors and
+                        solutions, so a dropped n, eps = 2^-24, a wrong norm or a
+                        transposed right-hand-side index changes the number
+                        (tests/test_oracle_checks.py)
+* ``metrics``           the SURVEY table's per-n numbers (test_oracle_checks.py)
+* ``spotrf_fig9_fp32``  debugging aid; integer-L0 exactness only.
 """
 from __future__ import annotations
 

@@ -16,6 +16,8 @@ import numpy as np
 EPS32 = 2.0 ** -23
 FACTOR_TOL = 1e-4
 RESID_TOL = 10.0
+STRICT_TOL = 1e-4        # R10 diagnostic bar: the north star's literal 1e-4 on kept entries
+STRICT_FLOOR = 1e-2      # entries >= STRICT_FLOOR * column max are kept
 
 
 def _mats(n, X, dtype=np.float64):
@@ -46,7 +48,7 @@ def colnorm_error(n, L_test, L64, info):
     return rel.max(axis=1) if n else np.zeros(len(info))
 
 
-def strict_relative_error(n, L_test, L64, info, floor=1e-2):
+def strict_relative_error(n, L_test, L64, info, floor=STRICT_FLOOR):
     """Diagnostic: elementwise relative error restricted to |L64_ij| >=
     floor * column max (R10's literal reading is ill-posed for entries that
     come from cancellation)."""
@@ -90,7 +92,10 @@ def upper_bits_unchanged(n, before, after):
 
 
 def accept(n, A_in, L_test, info_test, L64, info64):
-    """All of O1-O3 per matrix; returns dict of per-matrix arrays + ok mask."""
+    """All of O1-O3 per matrix; returns dict of per-matrix arrays + ok mask.
+    ``strict`` is the R10 diagnostic (elementwise relative error on entries
+    >= 1e-2 x column max); it is reported and checked separately against
+    STRICT_TOL by the parity tests, not folded into ``ok``."""
     info_test = np.asarray(info_test).reshape(-1)
     info64 = np.asarray(info64).reshape(-1)
     o1 = info_test == info64
@@ -99,7 +104,8 @@ def accept(n, A_in, L_test, info_test, L64, info64):
     ok_ok = info64 == 0
     o2 = e <= FACTOR_TOL
     o3 = np.where(ok_ok, r <= RESID_TOL, True)
-    return {"info_ok": o1, "err": e, "resid": np.where(ok_ok, r, 0.0),
+    strict = strict_relative_error(n, L_test, L64, info64)
+    return {"info_ok": o1, "err": e, "resid": np.where(ok_ok, r, 0.0), "strict": strict,
             "ok": o1 & o2 & o3}
 
 

@@ -51,6 +51,7 @@ def check_sample(n, batch, chunk, kind, dA, info, seed=2017, fail_period=0, uppe
     ginfo = info.cpu().numpy()[b]
     r = checks.accept(n, A, got, ginfo, L64, info64)
     assert r["ok"].all(), np.nonzero(~r["ok"])[0][:10]
+    assert r["strict"].max() <= checks.STRICT_TOL
     assert checks.upper_bits_unchanged(n, A, got).all()
     return got, b
 

@@ -77,3 +77,56 @@ def test_chunks_are_contiguous_and_coalesced():
                 assert (b // C) * C * n * n <= o < (b // C + 1) * C * n * n
                 if b % C != C - 1:
                     assert layout.offset(n, 256, C, b + 1, i, j) == o + 1
+
+
+# ---- right-hand-side (rectangular) layout, SURVEY §8(f) f1 -----------------
+# The n x nrhs block of matrix b is interleaved like the matrices (same chunk C):
+# element (i, r) at (b // C) * C * n * nrhs + (i + r * n) * C + b % C
+# (include/bspotrf.h, "Solves").  Offsets below are worked out by hand.
+
+def test_rect_offset_handworked():
+    # rows = 3, cols = 2, batch = 40, chunk 32: two chunks of 32 * 6 floats.
+    assert layout.rect_storage_elems(3, 2, 40, 32) == 2 * 32 * 6 == 384
+    assert layout.rect_offset(3, 2, 40, 32, 0, 0, 0) == 0
+    assert layout.rect_offset(3, 2, 40, 32, 5, 2, 0) == 2 * 32 + 5 == 69
+    assert layout.rect_offset(3, 2, 40, 32, 5, 0, 1) == 3 * 32 + 5 == 101
+    assert layout.rect_offset(3, 2, 40, 32, 33, 2, 1) == 192 + 5 * 32 + 1 == 353
+    # chunk 0: C = batch = 40, one chunk
+    assert layout.rect_storage_elems(3, 2, 40, 0) == 240
+    assert layout.rect_offset(3, 2, 40, 0, 33, 2, 1) == 5 * 40 + 33 == 233
+    assert layout.rect_offset(3, 2, 40, 0, 39, 0, 1) == 3 * 40 + 39 == 159
+    # cols = 1 (one right-hand side): a vector per matrix
+    assert layout.rect_offset(4, 1, 100, 64, 70, 3, 0) == 64 * 4 + 3 * 64 + 6 == 454
+    # empty problems
+    assert layout.rect_storage_elems(0, 2, 5, 32) == 0
+    assert layout.rect_storage_elems(3, 0, 5, 32) == 0
+    assert layout.rect_storage_elems(3, 2, 0, 32) == 0
+
+
+def test_rect_scatter_gather_handworked():
+    rows, cols, batch, chunk = 3, 2, 40, 32
+    b = np.arange(batch)[:, None]
+    e = np.arange(rows * cols)[None, :]
+    i, r = e % rows, e // rows
+    canon = (1000 * b + 10 * i + r).astype(np.float32)      # value names its (b, i, r)
+    out = layout.rect_to_interleaved(rows, cols, chunk, canon, fill_bits=0x7FC0DEAD)
+    assert out.size == 384
+    assert out[69] == 5020 and out[101] == 5001 and out[353] == 33021 and out[0] == 0
+    # pad lanes: matrices 40..63 of the second chunk, every element
+    for ee in range(6):
+        blk = out[192 + ee * 32 + 8:192 + (ee + 1) * 32]
+        assert (blk.view(np.uint32) == 0x7FC0DEAD).all()
+    assert (out.view(np.uint32) == 0x7FC0DEAD).sum() == 24 * 6
+    back = layout.rect_from_interleaved(rows, cols, batch, chunk, out)
+    assert np.array_equal(back, canon)
+    # a transposed (i, r) reading would put (b=5, i=0, r=1) at 1*32+5: it must not
+    assert out[1 * 32 + 5] == 5010
+
+
+@pytest.mark.parametrize("n,batch,chunk", [(5, 77, 32), (16, 70, 64), (3, 33, 0)])
+def test_rect_square_equals_matrix_layout(n, batch, chunk):
+    """rows == cols reduces to the matrix formula pinned by Fig. 10's walks."""
+    b = np.arange(batch)[:, None]
+    e = np.arange(n * n)[None, :]
+    assert np.array_equal(layout.rect_offset(n, n, batch, chunk, b, e % n, e // n),
+                          layout.offset(n, batch, chunk, b, e % n, e // n))
