@@ -27,7 +27,20 @@
  * launch.  No exceptions, no exit(), no printing.  Calls only ENQUEUE work on
  * `stream` (except batch_spotrf_interleaved_host, which is blocking); read
  * results after synchronising the stream.  No hidden allocation except in
- * batch_spotrf_interleaved_host.  Thread-safe and reentrant.
+ * batch_spotrf_interleaved_host, which takes its slab buffers from a
+ * library-owned cudaMemPool per device (created on first use, kept for reuse;
+ * the process's default pool is not touched).  Thread-safe and reentrant.
+ *
+ * TENSOR MEMORY.  Variants PTMEM, QTM, RCW and RCW16 (the table's choice for
+ * 24 <= n <= 64 at most chunks) allocate Tensor Memory per CTA with
+ * tcgen05.alloc and release it before the CTA exits; their shared-memory
+ * footprint caps the library's own demand at 512 columns per SM, so any number
+ * of concurrent launches of this library (any streams) make progress.
+ * tcgen05.alloc WAITS while the columns are held: a kernel from elsewhere that
+ * holds Tensor Memory on the same SM for an unbounded time (e.g. a persistent
+ * kernel that never relinquishes it) would stall these variants until it
+ * exits.  Such a process should select a non-TMEM variant explicitly through
+ * batch_spotrf_interleaved_ex (REG, SMEM, PANEL or TILE).
  * ----------------------------------------------------------------------------
  */
 #ifndef BSPOTRF_H

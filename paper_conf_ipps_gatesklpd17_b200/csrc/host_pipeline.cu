@@ -97,6 +97,35 @@ bool device_view(void *h, void **d) {
 // and each thread has its whole triangle's loads in flight, so both PCIe
 // directions stream at once).  TMA-staged variants are swapped for their
 // per-thread-load forms (the bulk engine is not used on host memory).
+// The library's own stream-ordered memory pool on the current device (one per
+// device, created on first use, never destroyed).  Its release threshold is
+// "keep everything", so the slab buffers of one host call are reused by the
+// next without a cudaMalloc; the process-wide default pool is left untouched.
+cudaError_t library_pool(cudaMemPool_t *out) {
+    static std::mutex mu;
+    static cudaMemPool_t pools[64] = {};
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (dev < 0 || dev >= 64) return cudaErrorInvalidDevice;
+    std::lock_guard<std::mutex> g(mu);
+    if (pools[dev] == nullptr) {
+        cudaMemPoolProps props = {};
+        props.allocType = cudaMemAllocationTypePinned;
+        props.handleTypes = cudaMemHandleTypeNone;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = dev;
+        cudaMemPool_t p = nullptr;
+        e = cudaMemPoolCreate(&p, &props);
+        if (e != cudaSuccess) return e;
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+        pools[dev] = p;
+    }
+    *out = pools[dev];
+    return cudaSuccess;
+}
+
 int zero_copy(int n, int64_t batch, int chunk, float *dA, int32_t *dinfo, int32_t *nfailed_out,
               cudaStream_t stream) {
     // Kernel choice for PCIe-resident data (scripts/zerocopy_probe.py on B200,
@@ -121,7 +150,9 @@ int zero_copy(int n, int64_t batch, int chunk, float *dA, int32_t *dinfo, int32_
         if (t.variant == BSPOTRF_VARIANT_PTMEM) t.staging = 2;
     }
     int32_t *dcount = nullptr;
-    cudaError_t e = cudaMallocAsync((void **)&dcount, sizeof(int32_t), stream);
+    cudaMemPool_t pool = nullptr;
+    cudaError_t e = library_pool(&pool);
+    if (e == cudaSuccess) e = cudaMallocFromPoolAsync((void **)&dcount, sizeof(int32_t), pool, stream);
     if (e != cudaSuccess) return (int)e;
     int rc = 0;
     e = cudaMemsetAsync(dcount, 0, sizeof(int32_t), stream);
@@ -194,24 +225,17 @@ extern "C" int batch_spotrf_interleaved_host(int n, int64_t batch, int chunk, fl
     BSP_TRY(cudaEventRecord(start, (cudaStream_t)stream));
     BSP_TRY(cudaStreamWaitEvent(sh, start, 0));
     {
-        static std::once_flag pool_once;  // keep freed slab buffers cached between calls
-        std::call_once(pool_once, [] {
-            int dev = 0;
-            cudaMemPool_t pool;
-            if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-                uint64_t thr = UINT64_MAX;
-                cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-            }
-        });
-    }
-    BSP_TRY(cudaMallocAsync((void **)&dcount, sizeof(int32_t), sh));
-    BSP_TRY(cudaMemsetAsync(dcount, 0, sizeof(int32_t), sh));
-    for (int i = 0; i < NS; ++i) {
-        BSP_TRY(cudaMallocAsync((void **)&slots[i].dA, (size_t)slab_elems * 4, sh));
-        BSP_TRY(cudaMallocAsync((void **)&slots[i].dinfo, (size_t)S * 4, sh));
-        BSP_TRY(cudaEventCreateWithFlags(&slots[i].h2d_done, cudaEventDisableTiming));
-        BSP_TRY(cudaEventCreateWithFlags(&slots[i].cmp_done, cudaEventDisableTiming));
-        BSP_TRY(cudaEventCreateWithFlags(&slots[i].d2h_done, cudaEventDisableTiming));
+        cudaMemPool_t pool = nullptr;
+        BSP_TRY(library_pool(&pool));
+        BSP_TRY(cudaMallocFromPoolAsync((void **)&dcount, sizeof(int32_t), pool, sh));
+        BSP_TRY(cudaMemsetAsync(dcount, 0, sizeof(int32_t), sh));
+        for (int i = 0; i < NS; ++i) {
+            BSP_TRY(cudaMallocFromPoolAsync((void **)&slots[i].dA, (size_t)slab_elems * 4, pool, sh));
+            BSP_TRY(cudaMallocFromPoolAsync((void **)&slots[i].dinfo, (size_t)S * 4, pool, sh));
+            BSP_TRY(cudaEventCreateWithFlags(&slots[i].h2d_done, cudaEventDisableTiming));
+            BSP_TRY(cudaEventCreateWithFlags(&slots[i].cmp_done, cudaEventDisableTiming));
+            BSP_TRY(cudaEventCreateWithFlags(&slots[i].d2h_done, cudaEventDisableTiming));
+        }
     }
     for (int64_t s = 0; s < nslabs; ++s) {
         Slot &sl = slots[s % NS];

@@ -107,6 +107,11 @@ potrf_rcw_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__r
         float *stg = unit(half, c);
         if constexpr (TMA) {
             if (threadIdx.x == 0) {
+                // the stage units were last written by the generic proxy (row
+                // buffer stores); the preceding __syncthreads orders the other
+                // threads' writes before this thread, the fence orders them
+                // before the async-proxy writes of the bulk copies
+                fence_proxy_async_smem();
                 const float *chunk = A + g * (int64_t)(32 * N * N);
                 mbar_arrive_expect_tx(&mbar[half], SH::bytes(c));
 #pragma unroll

@@ -89,6 +89,7 @@ potrf_rcw16_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *_
         float *stg = unit(half, c);
         if constexpr (TMA) {
             if (threadIdx.x == 0) {
+                fence_proxy_async_smem();        // generic RB stores -> async-proxy writes (see RCW)
                 const float *chunk = A + g * (int64_t)(32 * N * N);
                 mbar_arrive_expect_tx(&mbar[half], SH::bytes(c));
 #pragma unroll

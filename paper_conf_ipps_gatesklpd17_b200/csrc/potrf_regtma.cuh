@@ -27,9 +27,6 @@ __device__ __forceinline__ void bulk_s2g(void *dst, const void *src, uint32_t by
 }
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
-__device__ __forceinline__ void fence_proxy_async_smem() {
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-}
 
 // Resident CTAs per SM to ask ptxas for: as many as shared memory allows, but
 // never so many that fewer than T + 40 registers per thread would remain.
@@ -69,6 +66,7 @@ potrf_regtma_kernel(float *__restrict__ A, int32_t *__restrict__ info,
         for (int j = 0; j < N; ++j)
             bulk_g2s(img + tri<N>(j, j) * 32, chunk + (j + j * N) * 32, (uint32_t)((N - j) * 128), bar);
     }
+    __syncwarp();                                // barrier initialised before any lane polls it
     mbar_wait(bar, 0);
 
     float a[T];

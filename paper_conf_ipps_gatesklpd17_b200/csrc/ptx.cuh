@@ -36,6 +36,12 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
         : "memory");
 }
 
+// Order this thread's earlier generic-proxy accesses to shared memory before
+// later async-proxy (bulk copy) accesses of the same locations.
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
 // ---- TMA bulk copy global -> shared (1-D, 16-B granules) -------------------
 // Completes `bytes` of transaction count on `bar`.  dst, src 16-B aligned,
 // bytes a multiple of 16.  SASS: UBLKCP.

@@ -90,13 +90,33 @@ class RankBatch:
                       b0=self.b0, fail_seed=self.fail_seed, fail_period=self.fail_period,
                       stream=stream)
 
-    def factor(self, stream=None, tune=None):
-        """Factor this rank's slice; the count is accumulated on the device."""
+    def factor(self, stream=None, tune=None, reset=True):
+        """Factor this rank's slice (one kernel launch); the failure count is
+        accumulated on the device (``reset`` zeroes it first)."""
         from . import batch_spotrf_interleaved_ex
-        self.nfailed.zero_()
+        if reset:
+            self.nfailed.zero_()
         if self.count:
             batch_spotrf_interleaved_ex(self.n, self.count, self.chunk, self.A, self.info,
                                         nfailed=self.nfailed, tune=tune, stream=stream)
 
+    def reduce_failures(self, group=None):
+        """Enqueue the one collective (SUM of the 4-byte count) without a host
+        sync: after it, ``nfailed`` holds the global count on every rank."""
+        import torch.distributed as dist
+        if dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
+            dist.all_reduce(self.nfailed, op=dist.ReduceOp.SUM, group=group)
+
     def global_failures(self, group=None):
         return allreduce_count(self.nfailed, group)
+
+
+def min_over_ranks(value: int, device=None, group=None) -> int:
+    """The MIN over ranks of an integer (e.g. how many buffers fit in HBM), so
+    every rank runs the same number of steps and collectives pair up."""
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([int(value)], dtype=torch.int64, device=device)
+    if dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MIN, group=group)
+    return int(t.item())

@@ -51,3 +51,23 @@ def test_reference_arm_nonzero_rank_exits_quietly():
                           "--n", "4", "--batch", "100", "--steps", "1", "--warmup", "0"],
                          capture_output=True, text=True, timeout=300, cwd=ROOT, env=env)
     assert out.returncode == 0 and out.stdout.strip() == ""
+
+
+def test_default_workload_is_headline_config(monkeypatch):
+    """No flags -> BASELINE configs[2] (n=32, 4M, ALS, chunk 32): the largest
+    single-GPU config, the one the driver's bench line is quoted on."""
+    monkeypatch.setattr(sys, "argv", ["bench.py"])
+    a = bench.parse()
+    w = bench.workload(a)
+    assert (w["n"], w["batch"], w["chunk"], w["kind"]) == (32, 1 << 22, 32, "als")
+    assert "configs[2]" in w["desc"]
+    cfgs = json.load(open(os.path.join(ROOT, "BASELINE.json")))["configs"]
+    assert "n=32, batch=4M" in cfgs[2]
+    assert bench.parse_ns(a.per_n) == list(range(1, 65))
+    assert bench.parse_ns("1-3,8,16-17") == [1, 2, 3, 8, 16, 17]
+
+
+def test_host_budget_is_capped():
+    b = bench.host_budget_bytes(8)
+    assert 0 < b <= 48 << 30
+    assert bench.host_budget_bytes(1) >= b
