@@ -129,7 +129,24 @@ typedef struct {
     int staging;           /* SMEM/PANEL: 0 = auto, 1 = TMA bulk copy
                               (cp.async.bulk, needs chunk in {32,64,128}),
                               2 = per-thread cp.async                         */
+    int carveout;          /* preferred shared-memory carveout of the SM's
+                              unified L1/shared capacity, in percent (1..100;
+                              0 = driver default) -- Table I's "L1 or shared"
+                              parameter.  Applied to the
+                              kernel on every launch; the driver rounds it to a
+                              supported split and never grants less shared
+                              memory than the launch needs (a small carveout
+                              can lower the resident CTAs per SM).  Values
+                              outside 0..100 are rejected (-7).               */
 } bspotrf_tuning;
+
+/* 1 if the library holds a kernel instance for this explicit tuning at (n,
+ * chunk) -- i.e. batch_spotrf_interleaved_ex would not return -7 for want of
+ * an instance -- else 0; -1 n, -2 chunk invalid, -3 tune null.  The default
+ * build holds every instance the tuning table reaches plus a representative
+ * subset of the sweep space; BSPOTRF_SWEEP=1 at build time holds all of it
+ * (scripts/gen_instances.py).  No GPU work. */
+int bspotrf_tuning_available(int n, int chunk, const bspotrf_tuning *tune);
 
 /* Library version (major*10000 + minor*100 + patch). */
 int bspotrf_version(void);

@@ -21,7 +21,7 @@ __all__ = [
     "batch_spotrf_interleaved_host", "batch_spotrf_host_bytes",
     "bspotrf_synth_generate", "bspotrf_fill_u32", "bspotrf_probe_copy_lower", "Tuning",
     "batch_interleaved_rhs_elems", "batch_spotrs_interleaved", "batch_sposv_interleaved",
-    "VARIANT_AUTO", "VARIANT_REG", "VARIANT_SMEM", "VARIANT_TILE", "VARIANT_PANEL", "VARIANT_PTMEM", "VARIANT_RTMA", "VARIANT_RTMAP", "VARIANT_QTM", "VARIANT_REGX", "VARIANT_RCW", "VARIANT_REGV", "VARIANT_RCW16",
+    "bspotrf_tuning_available", "VARIANT_AUTO", "VARIANT_REG", "VARIANT_SMEM", "VARIANT_TILE", "VARIANT_PANEL", "VARIANT_PTMEM", "VARIANT_RTMA", "VARIANT_RTMAP", "VARIANT_QTM", "VARIANT_REGX", "VARIANT_RCW", "VARIANT_REGV", "VARIANT_RCW16",
     "SYNTH_KINDS", "UPPER_MODES", "LIB_PATH",
 ]
 
@@ -39,6 +39,7 @@ EXPORTS = (
     "batch_interleaved_to_canonical", "batch_spotrf_interleaved_host", "batch_spotrf_host_bytes",
     "bspotrf_synth_generate", "bspotrf_fill_u32", "bspotrf_probe_copy_lower",
     "batch_interleaved_rhs_elems", "batch_spotrs_interleaved", "batch_sposv_interleaved",
+    "bspotrf_tuning_available",
 )
 
 
@@ -53,7 +54,7 @@ class BspotrfError(RuntimeError):
 
 class Tuning(ctypes.Structure):
     _fields_ = [("variant", ctypes.c_int), ("threads_per_block", ctypes.c_int),
-                ("param", ctypes.c_int), ("staging", ctypes.c_int)]
+                ("param", ctypes.c_int), ("staging", ctypes.c_int), ("carveout", ctypes.c_int)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -69,6 +70,7 @@ _SIGS = {
     "batch_spotrf_interleaved": (_i32, [_i32, _i64, _i32, _vp, _vp, _vp]),
     "batch_spotrf_interleaved_ex": (_i32, [_i32, _i64, _i32, _vp, _vp, _vp, ctypes.POINTER(Tuning), _vp]),
     "bspotrf_get_tuning": (_i32, [_i32, _i32, ctypes.POINTER(Tuning)]),
+    "bspotrf_tuning_available": (_i32, [_i32, _i32, ctypes.POINTER(Tuning)]),
     "batch_canonical_to_interleaved": (_i32, [_i32, _i64, _i32, _vp, _vp, _vp]),
     "batch_interleaved_to_canonical": (_i32, [_i32, _i64, _i32, _vp, _vp, _vp]),
     "batch_spotrf_interleaved_host": (_i32, [_i32, _i64, _i32, _vp, _vp, _vp, _i64, _vp]),
@@ -153,6 +155,16 @@ def bspotrf_get_tuning(n: int, chunk: int) -> Tuning:
     t = Tuning()
     _check("bspotrf_get_tuning", lib().bspotrf_get_tuning(n, chunk, ctypes.byref(t)))
     return t
+
+
+def bspotrf_tuning_available(n: int, chunk: int, tune) -> bool:
+    """Whether the library holds a kernel instance for this explicit tuning."""
+    if isinstance(tune, dict):
+        tune = Tuning(**{k: int(v) for k, v in tune.items()})
+    rc = lib().bspotrf_tuning_available(n, chunk, ctypes.byref(tune))
+    if rc < 0:
+        raise BspotrfError("bspotrf_tuning_available", rc)
+    return rc == 1
 
 
 def batch_spotrf_interleaved(n, batch, chunk, A, info, stream=None):

@@ -177,8 +177,21 @@ extern "C" int bspotrf_get_tuning(int n, int chunk, bspotrf_tuning *out) {
         out->threads_per_block = 128;
         out->param = n <= 8 ? 4 : 8;
         out->staging = 0;
+        out->carveout = 0;
     }
     return 0;
+}
+
+extern "C" int bspotrf_tuning_available(int n, int chunk, const bspotrf_tuning *tune) {
+    const int rc = check_common(n, 1, chunk);
+    if (rc != 0) return rc;
+    if (tune == nullptr) return -3;
+    if (n == 0) return 1;
+    init_tables();
+    bspotrf_tuning t = *tune;
+    if (t.variant == BSPOTRF_VARIANT_AUTO) bspotrf_get_tuning(n, chunk, &t);
+    int tpb = 0;
+    return resolve(n, chunk, t, &tpb) != nullptr ? 1 : 0;
 }
 
 extern "C" int batch_spotrf_interleaved_ex(int n, int64_t batch, int chunk, float *A, int32_t *info,
@@ -196,6 +209,7 @@ extern "C" int batch_spotrf_interleaved_ex(int n, int64_t batch, int chunk, floa
         if (t.variant == BSPOTRF_VARIANT_AUTO) bspotrf_get_tuning(n, chunk, &t);
         if (t.threads_per_block < 0 || t.threads_per_block > 1024 || (t.threads_per_block % 32) != 0)
             return -7;
+        if (t.carveout < 0 || t.carveout > 100) return -7;
     } else {
         bspotrf_get_tuning(n, chunk, &t);
     }
@@ -216,6 +230,7 @@ extern "C" int batch_spotrf_interleaved_ex(int n, int64_t batch, int chunk, floa
     a.cstride = chunk > 0 ? chunk : batch;
     a.tpb = tpb;
     a.stream = (cudaStream_t)stream;
+    a.carveout = t.carveout;
     const cudaError_t e = fn(a);
     return e == cudaSuccess ? 0 : (int)e;
 }

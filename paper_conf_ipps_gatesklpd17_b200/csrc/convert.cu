@@ -36,7 +36,8 @@ constexpr int CV_PITCH = 33;
 struct CvShape {
     int64_t batch, C;
     int E, slices;          // slices = ceil(E / 32)
-    int64_t tiles;          // ceil(batch / 32) * slices
+    int64_t tiles;          // (ceil(batch / 32) - gbeg) * slices
+    int64_t gbeg;           // first 32-matrix group handled (the v2 kernel takes the full ones)
     int vec_i, vec_c;       // 128-bit interleaved / canonical accesses allowed
 };
 
@@ -48,8 +49,9 @@ struct CvTile {
 
 __device__ __forceinline__ CvTile cv_tile(const CvShape &s, int64_t t) {
     CvTile x;
-    const int64_t g = t / s.slices;
-    const int sl = (int)(t - g * s.slices);
+    const int64_t gt = t / s.slices;
+    const int sl = (int)(t - gt * s.slices);
+    const int64_t g = s.gbeg + gt;
     x.m0 = g * 32;
     x.ib = (x.m0 / s.C) * s.C * (int64_t)s.E + (x.m0 % s.C);
     x.e0 = sl * 32;
@@ -248,16 +250,351 @@ static cudaError_t launch_dir(const CvShape &s, const float *src, float *dst, cu
     return cudaGetLastError();
 }
 
+// ============================================================================
+// v2: 128-bit accesses on BOTH sides for every n (round 2; the v1 kernel above
+// used 32-bit canonical accesses for odd n -- 3.2-5.0 TB/s -- and wasted lanes
+// for n <= 4, where a 32-element tile holds E = n*n < 32 elements: 0.25-2.2 TB/s).
+// Preconditions: full 32-matrix groups only, C % 4 == 0 (interleaved lines
+// 16-B aligned), 16-B aligned bases; the v1 kernel takes the last partial group.
+//
+// A tile is P consecutive groups x an element slice [e0, e0 + es):
+//   path A (E <= 25, n <= 5; E compile-time): P = floor(33 / (E + 1)) whole
+//     groups -- on the canonical side ONE contiguous, 16-B aligned block of
+//     32*P*E floats (a group starts at 128*g*E bytes), moved as float4s;
+//   path B (E >= 36): P = 1, es <= ES (ES in {20,24,28,32}, slices balanced);
+//     canonical row m's segment [m*E + e0, +es) is moved through the aligned
+//     float4 "slots" covering it (phase = start % 4, 0 when E % 4 == 0): loads
+//     read whole slots (the few edge floats belong to a neighbouring tile and
+//     are discarded), stores write full slots with STG.128 and the (at most 2)
+//     edge slots per row with predicated scalar stores.
+// The interleaved side is pg*es lines of 32 floats (8 lanes x float4 per
+// line, 4 lines per warp instruction).  Each warp transposes through its own
+// [32P][ES+1] shared tile; the next tile's loads are in flight during the
+// current tile's stores (as v1).
+// ============================================================================
+constexpr int CV2_TILE = 32 * 33;            // floats of one warp's shared tile
+
+struct Cv2Shape {
+    int64_t C, G, tiles;   // chunk stride, full groups, tiles
+    int E, nsl, es_last;   // n*n, slices per group (B), width of the last slice (B)
+};
+
+__device__ __forceinline__ int64_t cv2_line(const Cv2Shape &s, int64_t g) {   // interleaved lane-0 offset
+    const int64_t m0 = g * 32;
+    return (m0 / s.C) * s.C * (int64_t)s.E + (m0 % s.C);
+}
+
+// ---- path A: E compile-time, P whole groups per tile ------------------------
+template <int E>
+struct Cv2A {
+    static constexpr int P = 33 / (E + 1);
+    static constexpr int PITCH = E + 1;
+    static constexpr int F4 = 8 * P * E;                 // float4s of a full tile's canonical block
+    static constexpr int LD = (F4 + 31) / 32;            // per lane
+    static constexpr int LINES = P * E;
+    static constexpr int LK = (LINES + 3) / 4;           // line steps per lane
+    // resident CTAs per SM to ask for: 3, or 2 where the held float4s
+    // (next tile's loads) would not fit 85 registers without spilling
+    static constexpr int MINB0 = LD >= 7 ? 2 : 3, MINB1 = LK >= 7 ? 2 : 3;
+};
+
+template <int DIR, int E>
+__global__ void __launch_bounds__(CV_THREADS, DIR == 0 ? Cv2A<E>::MINB0 : Cv2A<E>::MINB1)
+convert2a_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shape s) {
+    using SA = Cv2A<E>;
+    __shared__ float tiles[CV_WARPS][CV2_TILE];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    float *T = tiles[wid];
+    const int64_t W = (int64_t)gridDim.x * CV_WARPS;
+    int64_t t = (int64_t)blockIdx.x * CV_WARPS + wid;
+    if (t >= s.tiles) return;
+    const int c4 = (lane & 7) * 4, lq = lane >> 3;
+    float4 R[DIR == 0 ? SA::LD : SA::LK];
+    auto ngroups = [&](int64_t tt) {
+        const int64_t left = s.G - tt * SA::P;
+        return left < SA::P ? (int)left : SA::P;
+    };
+    auto load = [&](int64_t tt) {
+        const int64_t g0 = tt * SA::P;
+        const int pg = ngroups(tt);
+        if (DIR == 0) {                                   // canonical block, contiguous
+            const float *b = src + g0 * 32 * E;
+#pragma unroll
+            for (int k = 0; k < SA::LD; ++k) {
+                const int f = lane + 32 * k;
+                if (f < 8 * pg * E) R[k] = ldg4(b + 4 * f);
+            }
+        } else {                                          // interleaved lines
+#pragma unroll
+            for (int k = 0; k < SA::LK; ++k) {
+                const int li = 4 * k + lq;
+                if (li < pg * E) {
+                    const int gg = li / E, e = li - gg * E;
+                    R[k] = ldg4(src + cv2_line(s, g0 + gg) + (int64_t)e * s.C + c4);
+                }
+            }
+        }
+    };
+    load(t);
+    for (;;) {
+        const int pg = ngroups(t);
+        const int64_t g0 = t * SA::P;
+        if (DIR == 0) {
+#pragma unroll
+            for (int k = 0; k < SA::LD; ++k) {
+                const int f = lane + 32 * k;
+                if (f < 8 * pg * E) {
+                    const float v[4] = {R[k].x, R[k].y, R[k].z, R[k].w};
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const int x = 4 * f + j, m = x / E, e = x - m * E;
+                        T[m * SA::PITCH + e] = v[j];
+                    }
+                }
+            }
+        } else {
+#pragma unroll
+            for (int k = 0; k < SA::LK; ++k) {
+                const int li = 4 * k + lq;
+                if (li < pg * E) {
+                    const int gg = li / E, e = li - gg * E;
+                    const float v[4] = {R[k].x, R[k].y, R[k].z, R[k].w};
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) T[(32 * gg + c4 + j) * SA::PITCH + e] = v[j];
+                }
+            }
+        }
+        __syncwarp();
+        const int64_t tn = t + W;
+        const bool more = tn < s.tiles;
+        if (more) load(tn);
+        if (DIR == 0) {
+#pragma unroll
+            for (int k = 0; k < SA::LK; ++k) {
+                const int li = 4 * k + lq;
+                if (li < pg * E) {
+                    const int gg = li / E, e = li - gg * E;
+                    const float *r = T + (32 * gg + c4) * SA::PITCH + e;
+                    stg4(dst + cv2_line(s, g0 + gg) + (int64_t)e * s.C + c4, r[0], r[SA::PITCH],
+                         r[2 * SA::PITCH], r[3 * SA::PITCH]);
+                }
+            }
+        } else {
+            float *b = dst + g0 * 32 * E;
+#pragma unroll
+            for (int k = 0; k < SA::LD; ++k) {
+                const int f = lane + 32 * k;
+                if (f < 8 * pg * E) {
+                    float v[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const int x = 4 * f + j, m = x / E, e = x - m * E;
+                        v[j] = T[m * SA::PITCH + e];
+                    }
+                    stg4(b + 4 * f, v[0], v[1], v[2], v[3]);
+                }
+            }
+        }
+        if (!more) break;
+        __syncwarp();
+        t = tn;
+    }
+}
+
+// ---- path B: slices of ES elements, one group per tile ----------------------
+template <int ES, bool ALIGNED>
+struct Cv2B {
+    static constexpr int PITCH = ES + 1;
+    static constexpr int SL = ALIGNED ? ES / 4 : ES / 4 + 1;   // float4 slots per row
+    static constexpr int LD = (32 * SL + 31) / 32;             // per lane (== SL)
+    static constexpr int LK = ES / 4;                          // line steps per lane
+    static constexpr int MINB0 = LD >= 9 ? 2 : 3, MINB1 = LK >= 9 ? 2 : 3;
+};
+
+template <int DIR, int ES, bool ALIGNED>
+__global__ void __launch_bounds__(CV_THREADS, DIR == 0 ? Cv2B<ES, ALIGNED>::MINB0 : Cv2B<ES, ALIGNED>::MINB1)
+convert2b_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shape s) {
+    using SB = Cv2B<ES, ALIGNED>;
+    __shared__ float tiles[CV_WARPS][CV2_TILE];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    float *T = tiles[wid];
+    const int64_t W = (int64_t)gridDim.x * CV_WARPS;
+    int64_t t = (int64_t)blockIdx.x * CV_WARPS + wid;
+    if (t >= s.tiles) return;
+    const int c4 = (lane & 7) * 4, lq = lane >> 3;
+    float4 R[DIR == 0 ? SB::LD : SB::LK];
+    auto geom = [&](int64_t tt, int64_t &g, int &e0, int &es) {
+        g = tt / s.nsl;
+        const int sl = (int)(tt - g * s.nsl);
+        e0 = sl * ES;
+        es = sl == s.nsl - 1 ? s.es_last : ES;
+    };
+    auto load = [&](int64_t tt) {
+        int64_t g;
+        int e0, es;
+        geom(tt, g, e0, es);
+        if (DIR == 0) {                                   // canonical row segments via slots
+#pragma unroll
+            for (int k = 0; k < SB::LD; ++k) {
+                const int i = lane + 32 * k, r = i / SB::SL, sl = i - r * SB::SL;
+                const int64_t st = (g * 32 + r) * (int64_t)s.E + e0;
+                const int ph = ALIGNED ? 0 : (int)(st & 3);
+                if (r < 32 && 4 * sl < ph + es) R[k] = ldg4(src + (st - ph) + 4 * sl);
+            }
+        } else {
+            const int64_t base = cv2_line(s, g) + (int64_t)e0 * s.C + c4;
+#pragma unroll
+            for (int k = 0; k < SB::LK; ++k) {
+                const int li = 4 * k + lq;
+                if (li < es) R[k] = ldg4(src + base + (int64_t)li * s.C);
+            }
+        }
+    };
+    load(t);
+    for (;;) {
+        int64_t g;
+        int e0, es;
+        geom(t, g, e0, es);
+        if (DIR == 0) {
+#pragma unroll
+            for (int k = 0; k < SB::LD; ++k) {
+                const int i = lane + 32 * k, r = i / SB::SL, sl = i - r * SB::SL;
+                const int64_t st = (g * 32 + r) * (int64_t)s.E + e0;
+                const int ph = ALIGNED ? 0 : (int)(st & 3);
+                if (r < 32 && 4 * sl < ph + es) {
+                    const float v[4] = {R[k].x, R[k].y, R[k].z, R[k].w};
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const int idx = 4 * sl + j - ph;
+                        if (idx >= 0 && idx < es) T[r * SB::PITCH + idx] = v[j];
+                    }
+                }
+            }
+        } else {
+#pragma unroll
+            for (int k = 0; k < SB::LK; ++k) {
+                const int li = 4 * k + lq;
+                if (li < es) {
+                    const float v[4] = {R[k].x, R[k].y, R[k].z, R[k].w};
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) T[(c4 + j) * SB::PITCH + li] = v[j];
+                }
+            }
+        }
+        __syncwarp();
+        const int64_t tn = t + W;
+        const bool more = tn < s.tiles;
+        if (more) load(tn);
+        if (DIR == 0) {
+            const int64_t base = cv2_line(s, g) + (int64_t)e0 * s.C + c4;
+#pragma unroll
+            for (int k = 0; k < SB::LK; ++k) {
+                const int li = 4 * k + lq;
+                if (li < es) {
+                    const float *r = T + c4 * SB::PITCH + li;
+                    stg4(dst + base + (int64_t)li * s.C, r[0], r[SB::PITCH], r[2 * SB::PITCH], r[3 * SB::PITCH]);
+                }
+            }
+        } else {
+#pragma unroll
+            for (int k = 0; k < SB::LD; ++k) {
+                const int i = lane + 32 * k, r = i / SB::SL, sl = i - r * SB::SL;
+                const int64_t st = (g * 32 + r) * (int64_t)s.E + e0;
+                const int ph = ALIGNED ? 0 : (int)(st & 3);
+                if (r < 32 && 4 * sl < ph + es) {
+                    const int i0 = 4 * sl - ph;                  // element index of the slot's first float
+                    float *p = dst + (st - ph) + 4 * sl;
+                    if (i0 >= 0 && i0 + 4 <= es) {
+                        const float *q = T + r * SB::PITCH + i0;
+                        stg4(p, q[0], q[1], q[2], q[3]);
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < 4; ++j)
+                            if (i0 + j >= 0 && i0 + j < es) stg1(p + j, T[r * SB::PITCH + i0 + j]);
+                    }
+                }
+            }
+        }
+        if (!more) break;
+        __syncwarp();
+        t = tn;
+    }
+}
+
+template <typename K>
+static cudaError_t launch_persistent(K kern, int64_t tiles, const float *src, float *dst, const Cv2Shape &s,
+                                     cudaStream_t stream) {
+    int dev = 0, sms = 148, per_sm = 4;
+    if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, CV_THREADS, 0);
+    if (per_sm < 1) per_sm = 1;
+    int64_t grid = (int64_t)sms * per_sm;
+    const int64_t need = (tiles + CV_WARPS - 1) / CV_WARPS;
+    if (grid > need) grid = need;
+    if (grid < 1) grid = 1;
+    kern<<<(unsigned)grid, CV_THREADS, 0, stream>>>(src, dst, s);
+    return cudaGetLastError();
+}
+
+template <int DIR>
+static cudaError_t launch_v2(int n, int64_t G, int64_t C, const float *src, float *dst, cudaStream_t stream) {
+    Cv2Shape s;
+    s.C = C;
+    s.G = G;
+    s.E = n * n;
+    if (s.E <= 25) {
+        s.nsl = 1;
+        s.es_last = s.E;
+        switch (n) {
+#define BSP_CV2A(NN)                                                                       \
+    case NN: {                                                                             \
+        s.tiles = (G + Cv2A<NN * NN>::P - 1) / Cv2A<NN * NN>::P;                           \
+        return launch_persistent(convert2a_kernel<DIR, NN * NN>, s.tiles, src, dst, s, stream); \
+    }
+            BSP_CV2A(1) BSP_CV2A(2) BSP_CV2A(3) BSP_CV2A(4) BSP_CV2A(5)
+#undef BSP_CV2A
+        default:
+            return cudaErrorInvalidValue;
+        }
+    }
+    s.nsl = (s.E + 31) / 32;
+    const int per = (s.E + s.nsl - 1) / s.nsl;
+    const int ES = ((per + 3) / 4) * 4;                  // 20, 24, 28 or 32
+    s.nsl = (s.E + ES - 1) / ES;
+    s.es_last = s.E - (s.nsl - 1) * ES;
+    s.tiles = G * s.nsl;
+    const bool al = s.E % 4 == 0;
+#define BSP_CV2B(ESV)                                                                                    \
+    if (ES == ESV)                                                                                       \
+        return al ? launch_persistent(convert2b_kernel<DIR, ESV, true>, s.tiles, src, dst, s, stream)   \
+                  : launch_persistent(convert2b_kernel<DIR, ESV, false>, s.tiles, src, dst, s, stream);
+    BSP_CV2B(20) BSP_CV2B(24) BSP_CV2B(28) BSP_CV2B(32)
+#undef BSP_CV2B
+    return cudaErrorInvalidValue;
+}
+
 cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float *src, float *dst,
                            cudaStream_t stream) {
+    // 128-bit accesses need 16-B aligned bases (the ABI guarantees 16-B aligned pointers)
+    const bool al = ((uintptr_t)src % 16 == 0) && ((uintptr_t)dst % 16 == 0);
+    int64_t gbeg = 0;
+    if (al && C % 4 == 0) {                              // v2 for every full group
+        const int64_t G = batch / 32;
+        if (G > 0) {
+            const cudaError_t e = dir == 0 ? launch_v2<0>(n, G, C, src, dst, stream)
+                                           : launch_v2<1>(n, G, C, src, dst, stream);
+            if (e != cudaSuccess) return e;
+        }
+        gbeg = G;
+        if (G * 32 == batch) return cudaSuccess;
+    }
     CvShape s;
     s.batch = batch;
     s.C = C;
     s.E = n * n;
     s.slices = (s.E + 31) / 32;
-    s.tiles = ((batch + 31) / 32) * s.slices;
-    // 128-bit accesses need 16-B aligned bases (the ABI guarantees 16-B aligned pointers)
-    const bool al = ((uintptr_t)src % 16 == 0) && ((uintptr_t)dst % 16 == 0);
+    s.gbeg = gbeg;
+    s.tiles = ((batch + 31) / 32 - gbeg) * s.slices;
     s.vec_i = al && (C % 4 == 0);
     s.vec_c = al && (s.E % 4 == 0);
     if (dir == 0)

@@ -15,7 +15,21 @@ struct FactorArgs {
     int64_t cstride;     // effective chunk C (== batch for simple interleaved)
     int tpb;             // threads per block (multiple of 32)
     cudaStream_t stream;
+    int carveout = 0;    // preferred shared-memory carveout, percent (0 = driver default)
 };
+
+// Table I's "L1 or shared" axis (Sec. II.D): the
+// preferred split of the SM's unified L1 / shared-memory capacity, in percent
+// of the maximum shared memory, set on every launch (the attribute is per
+// function and persists, so a default launch must undo a tuned one).  0 is the
+// driver default (-1 to CUDA); the driver rounds to a supported configuration
+// and always grants at least what the launch needs.
+template <typename K>
+inline cudaError_t apply_carveout(K kern, int pct) {
+    return cudaFuncSetAttribute(reinterpret_cast<const void *>(kern),
+                                cudaFuncAttributePreferredSharedMemoryCarveout,
+                                pct <= 0 ? -1 : (pct > 100 ? 100 : pct));
+}
 
 using LaunchFn = cudaError_t (*)(const FactorArgs &);
 

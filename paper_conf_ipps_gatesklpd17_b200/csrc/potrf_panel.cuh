@@ -235,6 +235,7 @@ cudaError_t launch_panel(const FactorArgs &a) {
         const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
         if (e != cudaSuccess) return e;
     }
+    if (const cudaError_t ce = apply_carveout(kern, a.carveout); ce != cudaSuccess) return ce;
     kern<<<grid_for(a.batch, tpb), tpb, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
     return cudaGetLastError();
 }

@@ -418,6 +418,7 @@ cudaError_t launch_qtm(const FactorArgs &a) {
     auto kern = potrf_qtm_kernel<N, CT, P, COLS, PRE>;
     const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
+    if (const cudaError_t ce = apply_carveout(kern, a.carveout); ce != cudaSuccess) return ce;
     kern<<<grid_for(a.batch, SH::MPC), 128, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
     return cudaGetLastError();
 }

@@ -50,6 +50,16 @@ __device__ __forceinline__ void tmem_st8(uint32_t taddr, const float *v) {
                  : "memory");
 }
 
+// Row buffer, pair order: the four values v[kk] = L(8c+w, 4kq+kk) of row w are
+// stored so that float4 ((kq*4 + w/2)*2 + kk/2) of lane q holds
+// (L(w even, 2j), L(w odd, 2j), L(w even, 2j+1), L(w odd, 2j+1)), j = kk/2:
+// the reader's LDS.128 gives FFMA2 operand pairs over adjacent rows w, w+1.
+__device__ __forceinline__ void rb_put(float *rb, int kq, int w, int q, const float *v) {
+#pragma unroll
+    for (int kk = 0; kk < 4; ++kk)
+        rb[4 * (((kq * 4 + (w >> 1)) * 2 + (kk >> 1)) * 32 + q) + (kk & 1) * 2 + (w & 1)] = v[kk];
+}
+
 template <int N, int NCTA>
 struct RcwShape {
     static constexpr int W = 8;                          // column-block width = warps per CTA
@@ -173,31 +183,36 @@ potrf_rcw_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__r
             });
 
             // (b) acc(r) -= L(8r+h, 0..8c-1) L(8c..8c+7, 0..8c-1)^T, k ascending; the
-            //     rows of block c+1 (my slot c+1) are published to RB(c+1) on the way
+            //     rows of block c+1 (my slot c+1) are published to RB(c+1) on the way.
+            //     RB holds the b operand in pair order (rb_put) so that one LDS.128
+            //     yields (b[w][k], b[w+1][k]) register pairs for FFMA2 (f_upd2): two
+            //     columns w, w+1 of a row per instruction, the same bits as f_upd.
             if constexpr (c > 0) {
                 const float4 *rb = reinterpret_cast<const float4 *>(unit(half, 0)) + q;
-                float4 *rbn = reinterpret_cast<float4 *>(unit(half ^ 1, 0)) + h * 32 + q;
+                float *rbn = unit(half ^ 1, 0);
 #pragma unroll 1
                 for (int kq = 0; kq < 2 * c; ++kq) {
-                    float b[8][4];
+                    float4 x[4][2];                      // x[wp][j]: k = 2j, 2j+1 of rows 2wp, 2wp+1
 #pragma unroll
-                    for (int w = 0; w < 8; ++w) {
-                        const float4 x = rb[(kq * 8 + w) * 32];
-                        b[w][0] = x.x, b[w][1] = x.y, b[w][2] = x.z, b[w][3] = x.w;
-                    }
+                    for (int wp = 0; wp < 4; ++wp)
+#pragma unroll
+                        for (int j = 0; j < 2; ++j) x[wp][j] = rb[((kq * 4 + wp) * 2 + j) * 32];
                     float a[R][4];
                     sfor<c, R>([&](auto r_) {
                         constexpr int r = BSP_CI(r_);
                         tmem_ld4(tb + (uint32_t)(SH::off(r) + 4 * kq), a[r]);
                     });
                     tmem_wait_ld();
-                    if constexpr (c + 1 < R) rbn[kq * 256] = make_float4(a[c + 1][0], a[c + 1][1], a[c + 1][2], a[c + 1][3]);
+                    if constexpr (c + 1 < R) rb_put(rbn, kq, h, q, a[c + 1]);
                     sfor<c, R>([&](auto r_) {
                         constexpr int r = BSP_CI(r_);
 #pragma unroll
-                        for (int kk = 0; kk < 4; ++kk)
-#pragma unroll
-                            for (int w = 0; w < 8; ++w) acc[r][w] = f_upd(acc[r][w], a[r][kk], b[w][kk]);
+                        for (int wp = 0; wp < 4; ++wp) {
+                            f_upd2(acc[r][2 * wp], acc[r][2 * wp + 1], a[r][0], x[wp][0].x, x[wp][0].y);
+                            f_upd2(acc[r][2 * wp], acc[r][2 * wp + 1], a[r][1], x[wp][0].z, x[wp][0].w);
+                            f_upd2(acc[r][2 * wp], acc[r][2 * wp + 1], a[r][2], x[wp][1].x, x[wp][1].y);
+                            f_upd2(acc[r][2 * wp], acc[r][2 * wp + 1], a[r][3], x[wp][1].z, x[wp][1].w);
+                        }
                     });
                 }
             }
@@ -254,9 +269,8 @@ potrf_rcw_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__r
                 }
                 tmem_st8(tb + (uint32_t)(SH::off(r) + 8 * c), acc[r]);
                 if constexpr (r == c + 1) {
-                    float4 *rbn = reinterpret_cast<float4 *>(unit(half ^ 1, 0)) + h * 32 + q;
-                    rbn[(2 * c) * 256] = make_float4(acc[r][0], acc[r][1], acc[r][2], acc[r][3]);
-                    rbn[(2 * c + 1) * 256] = make_float4(acc[r][4], acc[r][5], acc[r][6], acc[r][7]);
+                    rb_put(unit(half ^ 1, 0), 2 * c, h, q, &acc[r][0]);
+                    rb_put(unit(half ^ 1, 0), 2 * c + 1, h, q, &acc[r][4]);
                 }
             });
             tmem_wait_st();
@@ -291,6 +305,7 @@ cudaError_t launch_rcw(const FactorArgs &a) {
     if (e != cudaSuccess) return e;
     const int64_t groups = (a.batch + 31) / 32;
     const int64_t grid = groups < (int64_t)nsm * NCTA ? groups : (int64_t)nsm * NCTA;
+    if (const cudaError_t ce = apply_carveout(kern, a.carveout); ce != cudaSuccess) return ce;
     kern<<<(unsigned)grid, 256, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
     return cudaGetLastError();
 }

@@ -286,6 +286,7 @@ cudaError_t launch_rcw16(const FactorArgs &a) {
     if (e != cudaSuccess) return e;
     const int64_t groups = (a.batch + 31) / 32;
     const int64_t grid = groups < (int64_t)nsm ? groups : (int64_t)nsm;
+    if (const cudaError_t ce = apply_carveout(kern, a.carveout); ce != cudaSuccess) return ce;
     kern<<<(unsigned)grid, 512, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride);
     return cudaGetLastError();
 }

@@ -71,6 +71,10 @@ template <int N, int CT, int MINW>
 cudaError_t launch_reg(const FactorArgs &a) {
     const int tpb = MINW ? 128 : (a.tpb > 0 ? a.tpb : 128);
     if (tpb > 256) return cudaErrorInvalidConfiguration;
+    {
+        auto kern = potrf_reg_kernel<N, CT, MINW>;
+        if (const cudaError_t ce = apply_carveout(kern, a.carveout); ce != cudaSuccess) return ce;
+    }
     potrf_reg_kernel<N, CT, MINW><<<grid_for(a.batch, tpb), tpb, 0, a.stream>>>(
         a.A, a.info, a.nfailed, a.batch, a.cstride);
     return cudaGetLastError();
@@ -162,6 +166,10 @@ cudaError_t launch_regx(const FactorArgs &a) {
     const int tpb = a.tpb > 0 ? a.tpb : 128;
     if (tpb > 128) return cudaErrorInvalidConfiguration;
     const int64_t per = (int64_t)tpb * M;
+    {
+        auto kern = potrf_regx_kernel<N, M, FAST>;
+        if (const cudaError_t ce = apply_carveout(kern, a.carveout); ce != cudaSuccess) return ce;
+    }
     potrf_regx_kernel<N, M, FAST><<<(unsigned)((a.batch + per - 1) / per), tpb, 0, a.stream>>>(
         a.A, a.info, a.nfailed, a.batch, a.cstride);
     return cudaGetLastError();

@@ -118,6 +118,7 @@ cudaError_t launch_regtma(const FactorArgs &a) {
         const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
         if (e != cudaSuccess) return e;
     }
+    if (const cudaError_t ce = apply_carveout(kern, a.carveout); ce != cudaSuccess) return ce;
     kern<<<grid_for(a.batch, W * 32), W * 32, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch);
     return cudaGetLastError();
 }
@@ -220,6 +221,7 @@ cudaError_t launch_rtmap(const FactorArgs &a) {
     int64_t grid = (int64_t)sms * per_sm;
     const int64_t need = (nchunks + W - 1) / W;
     if (grid > need) grid = need;
+    if (const cudaError_t ce = apply_carveout(kern, a.carveout); ce != cudaSuccess) return ce;
     kern<<<(unsigned)grid, W * 32, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch);
     return cudaGetLastError();
 }

@@ -91,6 +91,10 @@ cudaError_t launch_regv(const FactorArgs &a) {
     const int tpb = a.tpb > 0 ? a.tpb : 128;
     if (tpb > 128) return cudaErrorInvalidConfiguration;
     const int64_t groups = (a.batch + 3) / 4;
+    {
+        auto kern = potrf_regv_kernel<N>;
+        if (const cudaError_t ce = apply_carveout(kern, a.carveout); ce != cudaSuccess) return ce;
+    }
     potrf_regv_kernel<N><<<grid_for(groups, tpb), tpb, 0, a.stream>>>(a.A, a.info, a.nfailed, a.batch,
                                                                        a.cstride);
     return cudaGetLastError();

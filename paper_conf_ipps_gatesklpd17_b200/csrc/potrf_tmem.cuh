@@ -198,6 +198,15 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                     v[i + j * NB] = ok ? ld_stream(ad.at(m, c)) : 0.0f;
                 }
             tmem_st16(tbase + tidx(rb, pb), v);
+            // a warp barrier every FILL tiles keeps ptxas from hoisting every
+            // tile's loads above the first tcgen05.st: FILL*16 loads in flight
+            // (plus the register triangle's), no spills (round 2: n = 25, 29,
+            // 31 spilled 12-216 B, n = 33..42 up to 304 B, at 255 registers)
+            // (5 tiles with TMA staging; 1 with per-thread cp.async, whose address
+            // arithmetic for a runtime chunk stride needs the registers)
+            constexpr int idx = pb * TR - pb * (pb - 1) / 2 + (rb - pb);
+            constexpr int FILL = TMA ? 5 : 1;
+            if constexpr ((idx + 1) % FILL == 0) __syncwarp();
         });
     });
     tmem_wait_st();
@@ -327,10 +336,15 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
 #pragma unroll
                 for (int k = 0; k < NB; ++k)
 #pragma unroll
-                    for (int j = 0; j < NB; ++j)
+                    for (int j = 0; j < NB; ++j) {
+                        // rows i, i+1 in one FFMA2 (same bits as two f_upd)
 #pragma unroll
-                        for (int i = 0; i < ROWS; ++i)
-                            acc[i + j * NB] = f_upd(acc[i + j * NB], a[i + k * NB], b[j + k * NB]);
+                        for (int i = 0; i + 1 < ROWS; i += 2)
+                            f_upd2(acc[i + j * NB], acc[i + 1 + j * NB], b[j + k * NB], a[i + k * NB],
+                                   a[i + 1 + k * NB]);
+                        if constexpr (ROWS % 2 == 1)
+                            acc[ROWS - 1 + j * NB] = f_upd(acc[ROWS - 1 + j * NB], a[ROWS - 1 + k * NB], b[j + k * NB]);
+                    }
             });
             tmem_wait_ld();
 #pragma unroll
@@ -483,7 +497,8 @@ cudaError_t launch_ptmem(const FactorArgs &a) {
     const size_t floor_sm = SH::COLS == 256 ? 80 * 1024 : 120 * 1024;
     if (sm < floor_sm) sm = floor_sm;
     auto kern = potrf_ptmem_kernel<N, CT, S, TMA, false>;
-    const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e == cudaSuccess) e = apply_carveout(kern, a.carveout);
     if (e != cudaSuccess) return e;
     kern<<<grid_for(a.batch, 128), 128, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride,
                                                          nullptr);

@@ -14,11 +14,18 @@ Exhaustive over the B200 axes (north star (4)):
       RCW   8 warps per 32 matrices, CTAs per SM (1, 2), n > 32
       REGV  4 adjacent matrices per thread, 128-bit accesses, n <= 8
   * threads per block       -- 32..256
+  * L1 / shared carveout     -- --carveouts (percent of max shared memory; 0 =
+                               driver default): Table I's sixth parameter,
+                               PAPER.md:216,407
 Each point: regenerate the batch in place (device generator), flush L2, time
 ONE launch with CUDA events; median of --reps.  Every point is also checked
 (failure count 0 on SPD input).  Appends JSON lines (resumable).
 
     python scripts/autotune.py --n 1-32 --chunks 32,64,128,256,512,0 --out gpurun_out/sweep.jsonl
+
+The full candidate space needs the sweep build (BSPOTRF_SWEEP=1 python -m
+paper_conf_ipps_gatesklpd17_b200.build); the default build records the points
+it lacks as error -7.
 """
 import argparse
 import json
@@ -130,6 +137,9 @@ def main():
     ap.add_argument("--skip-from", action="append", default=[],
                     help="JSONL files whose points are already measured")
     ap.add_argument("--variants", default="1,2,3,4,5,6,7,8,10,11,12")   # 9 (REGX) on request
+    ap.add_argument("--carveouts", default="0", help="e.g. 0,1,25,50,100")
+    ap.add_argument("--only", default=None,
+                    help="JSON list of tunings to measure instead of candidates() (e.g. table rows)")
     a = ap.parse_args()
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     done = set()
@@ -137,8 +147,10 @@ def main():
         if os.path.exists(path):
             for line in open(path):
                 r = json.loads(line)
-                done.add((r["n"], r["chunk"], r["variant"], r["threads_per_block"], r["param"], r["staging"]))
+                done.add((r["n"], r["chunk"], r["variant"], r["threads_per_block"], r["param"], r["staging"],
+                          r.get("carveout", 0)))
     variants = {int(v) for v in a.variants.split(",")}
+    carveouts = [int(v) for v in a.carveouts.split(",")]
     dev = torch.device("cuda", 0)
     B = a.batch
     flush = torch.empty(512 << 18, dtype=torch.float32, device=dev)   # 512 MB > L2
@@ -152,10 +164,16 @@ def main():
             A = torch.empty(elems, dtype=torch.float32, device=dev)
             pristine = torch.empty_like(A)
             bsp.bspotrf_synth_generate(n, B, chunk, pristine, kind=a.kind, seed=2017)
-            for t in candidates(n, chunk):
+            cands = candidates(n, chunk)
+            if a.only:
+                cands = [dict(variant=t["variant"], threads_per_block=t["threads_per_block"],
+                              param=t["param"], staging=t["staging"])
+                         for t in json.loads(a.only) if t.get("n", n) == n and t.get("chunk", chunk) == chunk]
+            cands = [dict(t, carveout=cv) for t in cands for cv in carveouts]
+            for t in cands:
                 if t["variant"] not in variants:
                     continue
-                key = (n, chunk, t["variant"], t["threads_per_block"], t["param"], t["staging"])
+                key = (n, chunk, t["variant"], t["threads_per_block"], t["param"], t["staging"], t["carveout"])
                 if key in done:
                     continue
                 times = []

@@ -148,6 +148,63 @@ def sposv_ptmem_fits(n, s):
     return per_cta <= (100 * 1024 if cols == 256 else 220 * 1024)
 
 
+# ---- instance set: "core" (default) or the full sweep space -----------------
+# The full space (BSPOTRF_SWEEP=1) is every compile-time point the autotuning
+# sweep can visit (~1350 instances, ~12 min of nvcc on 8 cores, a 170 MB .so).
+# The default build keeps, for the variants with many panel widths / combos
+# (SMEM, PANEL, PTMEM, QTM, RTMAP), only what the tuning table (and the host
+# pipeline's zero-copy choice) can reach plus one representative point per n,
+# which the parity and bit-identity tests cover; every other variant is cheap
+# and is always built whole.  Tests ask bspotrf_tuning_available() before
+# running an explicit tuning.
+SWEEP = os.environ.get("BSPOTRF_SWEEP", "0") not in ("", "0")
+
+
+def _table_params():
+    """{(variant, n): set of param (panel width / P), plus QTM staging codes}."""
+    out = {}
+    try:
+        for r in json.load(open(TABLE))["entries"]:
+            out.setdefault((r["variant"], r["n"]), set()).add((r["param"], r["staging"]))
+    except FileNotFoundError:
+        pass
+    return out
+
+
+def zero_copy_panel_s(n):
+    """Panel width the host pipeline's zero-copy path picks for 20 < n <= 32
+    (csrc/host_pipeline.cu zero_copy)."""
+    s = ((n - 16 + 3) // 4) * 4 if n - 16 >= 4 else 4
+    if n - s > 16 or s > n - 8:
+        s = ((n - 12) // 4) * 4
+    return s
+
+
+def keep(variant, n, param, staging=None, table=None):
+    if SWEEP:
+        return True
+    tp = (table or {}).get((variant, n), set())
+    if variant == 8:                              # QTM: (P, staging code)
+        combos = [(p, qtm_staging(c, pre)) for p, c, pre in QTM_COMBOS if qtm_fits(n, p, c, pre)]
+        return (param, staging) in tp or (combos and (param, staging) == combos[0])
+    if variant == 7:                              # RTMAP (a measured negative result)
+        return param == 2
+    table_s = {p for p, _ in tp}
+    if param in table_s:
+        return True
+    if variant == 2:
+        vals = smem_s_values(n)
+        rep = n - 14 if (n - 14) in vals else (vals[0] if vals else None)
+        return param == rep
+    if variant == 4:
+        vals = panel_s_values(n)
+        return param == (vals[0] if vals else None) or (20 < n <= 32 and param == zero_copy_panel_s(n))
+    if variant == 5:
+        vals = ptmem_s_values(n)
+        return param == (vals[0] if vals else None)
+    return True
+
+
 def write_if_changed(path, text):
     if os.path.exists(path) and open(path).read() == text:
         return False
@@ -158,6 +215,7 @@ def write_if_changed(path, text):
 
 def main():
     os.makedirs(GEN, exist_ok=True)
+    table = _table_params()
     entries = []
     files = set()
     hdr = "// GENERATED by scripts/gen_instances.py -- do not edit\n"
@@ -173,6 +231,8 @@ def main():
         files.add(name)
     for n in SMEM_N:
         for s in smem_s_values(n):
+            if not keep(2, n, s, table=table):
+                continue
             body = [hdr, '#include "../potrf_smem.cuh"', "namespace bsp {"]
             for ct, tma in SMEM_COMBOS:
                 t = "true" if tma else "false"
@@ -184,6 +244,8 @@ def main():
             files.add(name)
     for n in PANEL_N:
         for s in panel_s_values(n):
+            if not keep(4, n, s, table=table):
+                continue
             body = [hdr, '#include "../potrf_panel.cuh"', "namespace bsp {"]
             for ct, tma in SMEM_COMBOS:
                 t = "true" if tma else "false"
@@ -198,8 +260,9 @@ def main():
         for w in RTMA_W:
             body.append(f"template cudaError_t launch_regtma<{n}, {w}>(const FactorArgs &);")
             entries.append(f"{{6, {n}, {w}, 32, 1, &launch_regtma<{n}, {w}>}}")
-            body.append(f"template cudaError_t launch_rtmap<{n}, {w}>(const FactorArgs &);")
-            entries.append(f"{{7, {n}, {w}, 32, 1, &launch_rtmap<{n}, {w}>}}")
+            if keep(7, n, w, table=table):
+                body.append(f"template cudaError_t launch_rtmap<{n}, {w}>(const FactorArgs &);")
+                entries.append(f"{{7, {n}, {w}, 32, 1, &launch_rtmap<{n}, {w}>}}")
         body.append("}  // namespace bsp\n")
         name = f"inst_rtma_{n:02d}.cu"
         write_if_changed(os.path.join(GEN, name), "\n".join(body))
@@ -207,6 +270,8 @@ def main():
     sposv_ptmem_entries = []
     for n in PTMEM_N:
         for s in ptmem_s_values(n):
+            if not keep(5, n, s, table=table):
+                continue
             body = [hdr, '#include "../potrf_tmem.cuh"', "namespace bsp {"]
             for ct, tma in PTMEM_COMBOS:
                 t = "true" if tma else "false"
@@ -233,7 +298,7 @@ def main():
     for n in QTM_N:
         body = [hdr, '#include "../potrf_qtm.cuh"', "namespace bsp {"]
         for p, cols, pre in QTM_COMBOS:
-            if not qtm_fits(n, p, cols, pre):
+            if not qtm_fits(n, p, cols, pre) or not keep(8, n, p, qtm_staging(cols, pre), table=table):
                 continue
             pr = "true" if pre else "false"
             for ct in QTM_CT:
@@ -318,11 +383,13 @@ def main():
     rows = [hdr, f"// source: tuning/table.json ({table.get('source', '?')})",
             "static const TuneEntry kTuning[] = {"]
     for r in table["entries"]:
-        rows.append("    {%d, %d, {%d, %d, %d, %d}}," % (
-            r["n"], r["chunk"], r["variant"], r["threads_per_block"], r["param"], r["staging"]))
+        rows.append("    {%d, %d, {%d, %d, %d, %d, %d}}," % (
+            r["n"], r["chunk"], r["variant"], r["threads_per_block"], r["param"], r["staging"],
+            r.get("carveout", 0)))
     rows.append("};\n")
     write_if_changed(os.path.join(GEN, "tuning_table.inc"), "\n".join(rows))
-    print(f"{len(files)} instance files, {len(entries)} instances, {len(table['entries'])} tuning rows")
+    print(f"{len(files)} instance files, {len(entries)} instances ({'full sweep space' if SWEEP else 'core set'}), "
+          f"{len(table['entries'])} tuning rows")
 
 
 if __name__ == "__main__":

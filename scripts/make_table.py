@@ -20,7 +20,7 @@ for r in ok:
         best[k] = r
 def key(r):
     return dict(variant=r["variant"], threads_per_block=r["threads_per_block"], param=r["param"],
-                staging=r["staging"])
+                staging=r["staging"], carveout=r.get("carveout", 0))
 entries = []
 ns = sorted({r["n"] for r in ok})
 for n in ns:

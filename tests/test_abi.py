@@ -107,6 +107,24 @@ def test_explicit_tuning_rejects_unavailable(L):
     assert L.batch_spotrf_interleaved_ex(20, 10, 32, fake, fake, None, ctypes.byref(t), None) == -7
     t = bsp.Tuning(bsp.VARIANT_REG, 48, 0, 0)     # tpb not a multiple of 32
     assert L.batch_spotrf_interleaved_ex(8, 10, 32, fake, fake, None, ctypes.byref(t), None) == -7
+    t = bsp.Tuning(bsp.VARIANT_REG, 128, 0, 0, 101)   # carveout outside 0..100 percent
+    assert L.batch_spotrf_interleaved_ex(8, 10, 32, fake, fake, None, ctypes.byref(t), None) == -7
+    t = bsp.Tuning(bsp.VARIANT_REG, 128, 0, 0, -1)
+    assert L.batch_spotrf_interleaved_ex(8, 10, 32, fake, fake, None, ctypes.byref(t), None) == -7
+
+
+def test_tuning_struct_matches_header():
+    """bspotrf_tuning in include/bspotrf.h: five ints, carveout last (Table I's
+    L1/shared parameter); the table's rows all use the driver default or a
+    percentage."""
+    hdr = open(os.path.join(ROOT, "include", "bspotrf.h")).read()
+    body = hdr[hdr.index("typedef struct {", hdr.index("Launch tuning")):hdr.index("} bspotrf_tuning;")]
+    fields = re.findall(r"^\s*int\s+(\w+);", body, flags=re.M)
+    assert fields == [f for f, _ in bsp.Tuning._fields_] == \
+        ["variant", "threads_per_block", "param", "staging", "carveout"]
+    for n in range(1, 65):
+        for chunk in (0, 32, 64, 96):
+            assert 0 <= bsp.bspotrf_get_tuning(n, chunk).carveout <= 100
 
 
 def test_product_never_imports_oracle():
@@ -122,3 +140,17 @@ def test_product_never_imports_oracle():
         assert "paper_conf_ipps_gatesklpd17_b200" not in txt.replace(
             "paper_conf_ipps_gatesklpd17_b200/csrc", "").replace(
             "(``paper_conf_ipps_gatesklpd17_b200``)", ""), f
+
+
+def test_every_table_choice_is_built():
+    """The default (core) build must hold the instance of every tuning-table
+    row it can reach, for every n and chunk class (host logic, no GPU)."""
+    for n in range(1, 65):
+        for chunk in (0, 32, 64, 96, 128, 256, 512, 1024):
+            t = bsp.bspotrf_get_tuning(n, chunk)
+            assert bsp.bspotrf_tuning_available(n, chunk, t), (n, chunk, t.as_dict())
+    # an explicit tuning with no instance is reported, not launched
+    assert not bsp.bspotrf_tuning_available(40, 32, dict(variant=bsp.VARIANT_REG, threads_per_block=128,
+                                                         param=0, staging=0))
+    with pytest.raises(bsp.BspotrfError):
+        bsp.bspotrf_tuning_available(65, 32, dict(variant=1, threads_per_block=0, param=0, staging=0))

@@ -12,13 +12,17 @@ from gpu_helpers import assert_parity, make_batch, run_gpu, torch_mod
 pytestmark = pytest.mark.gpu
 
 
-@pytest.mark.parametrize("n", [1, 2, 3, 5, 8, 16, 31, 32, 64])
+@pytest.mark.parametrize("n", [1, 2, 3, 4, 5, 6, 7, 8, 9, 12, 16, 31, 32, 33, 45, 63, 64])
 @pytest.mark.parametrize("chunk", [32, 64, 0, 160])
-@pytest.mark.parametrize("batch", [517, 1024, 96, 1])
+@pytest.mark.parametrize("batch", [517, 1024, 96, 1, 1184, 1002])
 def test_conversion_matches_layout_definition(n, chunk, batch):
-    """batch 517: ragged last group (32-bit interleaved accesses, masked); 1024 and
-    96 with chunk 0: C % 4 == 0 (128-bit interleaved path); even n: 128-bit
-    canonical path; odd n: 32-bit canonical path (rows not 16-B aligned)."""
+    """The v2 kernel (128-bit on both sides) takes every full 32-matrix group
+    when C % 4 == 0: n <= 5 as whole-group blocks (path A, several groups per
+    tile, a partial last block at batch 1184 = 37 groups), n >= 6 as balanced
+    element slices with aligned float4 slots (path B; odd n: phase != 0, edge
+    slots stored by scalars).  The v1 kernel takes the ragged last group
+    (batch 517, 1002) and chunk 0 with batch % 4 != 0 (1002: 32-bit
+    interleaved accesses); batch 1: v1 only."""
     torch = torch_mod()
     rng = np.random.default_rng(n * 1000 + chunk)
     canon = rng.standard_normal((batch, n * n)).astype(np.float32)

@@ -97,10 +97,11 @@ def test_qtm_parity_failures_ragged(n, chunk):
     canon, inter = make_batch(n, batch, chunk, kind="dd", seed=n, fail_seed=2018, fail_period=5)
     failed, kk = synth.fail_plan(n, 2018, 5, np.arange(batch, dtype=np.uint64))
     combos = _qtm_combos(n)
-    assert combos
-    for p_, cols, pre in combos:
-        t = dict(variant=bsp.VARIANT_QTM, threads_per_block=128, param=p_,
-                 staging=gen_instances_mod().qtm_staging(cols, pre))
+    ts = [dict(variant=bsp.VARIANT_QTM, threads_per_block=128, param=p_,
+               staging=gen_instances_mod().qtm_staging(cols, pre)) for p_, cols, pre in combos]
+    ts = [t for t in ts if bsp.bspotrf_tuning_available(n, chunk, t)]
+    assert ts                                      # the core build keeps one QTM point per n
+    for t in ts:
         out, info, cnt = run_gpu(n, batch, chunk, inter, tune=t)
         assert np.array_equal(info, np.where(failed, kk + 1, 0)), t
         assert_parity(n, batch, chunk, canon, inter, out, info, cnt)
@@ -225,7 +226,9 @@ def _tunings(n, chunk):
                 out.append(dict(variant=bsp.VARIANT_SMEM, threads_per_block=64, param=s, staging=2))
                 if chunk in (32, 64, 128):
                     out.append(dict(variant=bsp.VARIANT_SMEM, threads_per_block=0, param=s, staging=1))
-    return out
+    # the default (core) build holds a subset of the sweep space: test every
+    # instance it has (BSPOTRF_SWEEP=1 builds all of them)
+    return [t for t in out if bsp.bspotrf_tuning_available(n, chunk, t)]
 
 
 @pytest.mark.parametrize("n", [2, 7, 13, 16, 19, 20, 21, 23, 24, 25, 27, 28, 29, 30, 31, 32, 33, 36, 39,
@@ -236,7 +239,12 @@ def test_all_variants_bitwise_identical(n, chunk):
     batch = 2 * 128 + 19
     canon, inter = make_batch(n, batch, chunk, kind="als", seed=77)
     ref = None
-    for t in _tunings(n, chunk):
+    ts = _tunings(n, chunk)
+    table = bsp.bspotrf_get_tuning(n, chunk).as_dict()
+    variants = {t["variant"] for t in ts}
+    assert len(ts) >= 3 and len(variants) >= 2, ts
+    ts.append(table)                               # the table's own choice, whatever it is
+    for t in ts:
         out, info, cnt = run_gpu(n, batch, chunk, inter, tune=t)
         if ref is None:
             assert_parity(n, batch, chunk, canon, inter, out, info, cnt)
