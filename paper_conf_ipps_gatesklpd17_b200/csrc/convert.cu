@@ -276,7 +276,7 @@ constexpr int CV2_TILE = 32 * 33;            // floats of one warp's shared tile
 
 struct Cv2Shape {
     int64_t C, G, tiles;   // chunk stride, full groups, tiles
-    int E, nsl, es_last;   // n*n, slices per group (B), width of the last slice (B)
+    int E, nsl, esw, es_last;   // n*n; path B: slices per group, slice width (<= ES), last slice
 };
 
 __device__ __forceinline__ int64_t cv2_line(const Cv2Shape &s, int64_t g) {   // interleaved lane-0 offset
@@ -426,8 +426,13 @@ convert2b_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
     auto geom = [&](int64_t tt, int64_t &g, int &e0, int &es) {
         g = tt / s.nsl;
         const int sl = (int)(tt - g * s.nsl);
-        e0 = sl * ES;
-        es = sl == s.nsl - 1 ? s.es_last : ES;
+        if (ALIGNED) {                                    // float4-aligned slice starts
+            e0 = sl * s.esw;
+            es = sl == s.nsl - 1 ? s.es_last : s.esw;
+        } else {                                          // proportional: widths differ by <= 1
+            e0 = (int)((int64_t)sl * s.E / s.nsl);
+            es = (int)((int64_t)(sl + 1) * s.E / s.nsl) - e0;
+        }
     };
     auto load = [&](int64_t tt) {
         int64_t g;
@@ -545,6 +550,7 @@ static cudaError_t launch_v2(int n, int64_t G, int64_t C, const float *src, floa
     if (s.E <= 25) {
         s.nsl = 1;
         s.es_last = s.E;
+        s.esw = s.E;
         switch (n) {
 #define BSP_CV2A(NN)                                                                       \
     case NN: {                                                                             \
@@ -558,9 +564,13 @@ static cudaError_t launch_v2(int n, int64_t G, int64_t C, const float *src, floa
         }
     }
     s.nsl = (s.E + 31) / 32;
-    const int per = (s.E + s.nsl - 1) / s.nsl;
-    const int ES = ((per + 3) / 4) * 4;                  // 20, 24, 28 or 32
-    s.nsl = (s.E + ES - 1) / ES;
+    const int per = (s.E + s.nsl - 1) / s.nsl;           // balanced slices of <= 32 elements
+    const int ES = ((per + 3) / 4) * 4;                  // buffer width: 20, 24, 28 or 32
+    // aligned rows (E % 4 == 0) keep slice starts on float4 boundaries; otherwise
+    // slices are cut proportionally in the kernel (widths per-1 or per, no
+    // near-empty tail slice, e.g. E = 961, 1089, 3969)
+    s.esw = ES;
+    if (s.E % 4 == 0) s.nsl = (s.E + ES - 1) / ES;
     s.es_last = s.E - (s.nsl - 1) * ES;
     s.tiles = G * s.nsl;
     const bool al = s.E % 4 == 0;
@@ -578,7 +588,13 @@ cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float
     // 128-bit accesses need 16-B aligned bases (the ABI guarantees 16-B aligned pointers)
     const bool al = ((uintptr_t)src % 16 == 0) && ((uintptr_t)dst % 16 == 0);
     int64_t gbeg = 0;
-    if (al && C % 4 == 0) {                              // v2 for every full group
+    // v2 for every full group -- except interleaved -> canonical at odd n >= 7
+    // (path B with phase != 0): there its edge slots (predicated scalar stores,
+    // 4 scalar LDS per slot) measured 2.6-3.5 TB/s against v1's 3.2-3.7
+    // (profiles/r02/ncu_convert.md: mio_throttle + short_scoreboard bound).
+    const int E = n * n;
+    const bool v2 = al && C % 4 == 0 && !(dir == 1 && E > 25 && E % 4 != 0);
+    if (v2) {
         const int64_t G = batch / 32;
         if (G > 0) {
             const cudaError_t e = dir == 0 ? launch_v2<0>(n, G, C, src, dst, stream)

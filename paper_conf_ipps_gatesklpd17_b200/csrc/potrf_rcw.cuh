@@ -190,13 +190,14 @@ potrf_rcw_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__r
             if constexpr (c > 0) {
                 const float4 *rb = reinterpret_cast<const float4 *>(unit(half, 0)) + q;
                 float *rbn = unit(half ^ 1, 0);
-#pragma unroll 1
-                for (int kq = 0; kq < 2 * c; ++kq) {
-                    float4 x[4][2];                      // x[wp][j]: k = 2j, 2j+1 of rows 2wp, 2wp+1
+                // b operand of k-chunk kq: x[wp][j] = k 4kq+2j, 4kq+2j+1 of rows 2wp, 2wp+1
+                auto ldb = [&](float4 (&x)[4][2], int kq) {
 #pragma unroll
                     for (int wp = 0; wp < 4; ++wp)
 #pragma unroll
                         for (int j = 0; j < 2; ++j) x[wp][j] = rb[((kq * 4 + wp) * 2 + j) * 32];
+                };
+                auto step = [&](const float4 (&x)[4][2], int kq) {
                     float a[R][4];
                     sfor<c, R>([&](auto r_) {
                         constexpr int r = BSP_CI(r_);
@@ -214,6 +215,12 @@ potrf_rcw_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__r
                             f_upd2(acc[r][2 * wp], acc[r][2 * wp + 1], a[r][3], x[wp][1].z, x[wp][1].w);
                         }
                     });
+                };
+#pragma unroll 1
+                for (int kq = 0; kq < 2 * c; ++kq) {
+                    float4 x[4][2];
+                    ldb(x, kq);
+                    step(x, kq);
                 }
             }
 

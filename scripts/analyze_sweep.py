@@ -37,9 +37,13 @@ def main():
     from sklearn.model_selection import train_test_split
 
     rows = load(sys.argv[1:])
-    feats = ["n", "variant", "chunking", "chunk size", "threads/block", "panel or tile width", "staging"]
+    feats = ["n", "variant", "chunking", "chunk size", "threads/block", "panel or tile width", "staging",
+             "L1/shared carveout"]
+    # carveout: percent of max shared memory preferred (0 = driver default); points
+    # without the field were measured at the default (round-1 sweep)
     X = np.array([[r["n"], r["variant"], int(r["chunk"] > 0), r["chunk"] if r["chunk"] > 0 else 0,
-                   r["threads_per_block"], r["param"], r["staging"]] for r in rows], dtype=float)
+                   r["threads_per_block"], r["param"], r["staging"], r.get("carveout", 0)] for r in rows],
+                 dtype=float)
     y = np.array([r["gflops"] for r in rows])
     Xtr, Xte, ytr, yte = train_test_split(X, y, test_size=0.25, random_state=2017)
     rf = RandomForestRegressor(n_estimators=500, random_state=2017, n_jobs=-1, oob_score=True)
@@ -64,11 +68,32 @@ def main():
           f"correlation r = {corr:.4f} (the paper's Fig. 21).\n")
     print("| Parameter | %IncMSE (permutation, held-out 25%) | Type |")
     print("|---|---|---|")
-    types = ["integer", "categorical (6)", "binary", "integer", "integer", "integer", "categorical (3)"]
+    types = ["integer", "categorical (12)", "binary", "integer", "integer", "integer", "categorical (3)",
+             "integer (0 = default, 1..100 %)"]
     for f, v, t in sorted(zip(feats, imp, types), key=lambda x: -x[1]):
         print(f"| {f} | {v:.1f} | {t} |")
     print("\nPaper Table I (P100, for comparison): n 43.1; tile size 103.9; looking 99.9; "
           "chunking 157.4; chunk size 25.9; unrolling 85.7; L1/shared -18.6.")
+    carve = [r for r in rows if r.get("carveout", 0) != 0]
+    if carve:
+        import collections
+        by = collections.defaultdict(dict)
+        for r in rows:
+            if r.get("batch", 1 << 20) == 1 << 20:
+                by[(r["n"], r["chunk"], r["variant"], r["threads_per_block"], r["param"], r["staging"])][
+                    r.get("carveout", 0)] = r["gbs"]
+        print("\n## Carveout axis (the tuning table's kernel at each n, 1M matrices)\n")
+        print("GB/s at each preferred shared-memory carveout (percent of max shared memory; "
+              "default = driver's choice).\n")
+        print("| n | chunk | variant | default | 1% | 25% | 50% | 100% | best / default |")
+        print("|---|---|---|---|---|---|---|---|---|")
+        V = {1: "REG", 2: "SMEM", 3: "TILE", 4: "PANEL", 5: "PTMEM", 6: "RTMA", 7: "RTMAP", 8: "QTM",
+             9: "REGX", 10: "RCW", 11: "REGV", 12: "RCW16"}
+        for k, d in sorted(by.items()):
+            if len(d) < 5:
+                continue
+            cells = " | ".join(f"{d.get(c, float('nan')):.0f}" for c in (0, 1, 25, 50, 100))
+            print(f"| {k[0]} | {k[1]} | {V[k[2]]} | {cells} | {max(d.values()) / d[0]:.3f} |")
 
 
 if __name__ == "__main__":

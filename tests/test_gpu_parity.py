@@ -281,3 +281,42 @@ def test_nan_pivot_reported():
     out, info, cnt = run_gpu(n, batch, 32, inter)
     assert info[5] == 4 and info[9] == 1 and cnt == 2
     assert (np.delete(info, [5, 9]) == 0).all()
+
+
+@pytest.mark.parametrize("n", [40, 57, 64])
+@pytest.mark.parametrize("chunk", [32, 0, 96])
+def test_rcw_many_groups_per_cta(n, chunk):
+    """RCW / RCW16 are persistent (one or two CTAs per SM): with more than
+    2 * SMs * 32 matrices every CTA loops over several 32-matrix groups, so the
+    next-group prefetch, the half flip and the mbarrier parity across groups
+    are exercised, with a ragged tail.  Sampled matrices against the oracle
+    (first/last groups of every CTA's walk are in the sample), the fused count
+    exact, and RCW == RCW16 bitwise (P8)."""
+    torch = torch_mod()
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    batch = 2 * sms * 32 * 3 + 77
+    b = np.arange(batch, dtype=np.uint64)
+    canon = synth.generate(n, "dd", 31, b, upper="nan", fail_seed=2018, fail_period=97)
+    failed, kk = synth.fail_plan(n, 2018, 97, b)
+    inter = layout.to_interleaved(n, chunk, canon, fill_bits=synth.PAD_BITS)
+    ts = [dict(variant=bsp.VARIANT_RCW, threads_per_block=256, param=k, staging=0) for k in _rcw_ncta(n)]
+    if n in gen_instances_mod().RCW16_N:
+        ts.append(dict(variant=bsp.VARIANT_RCW16, threads_per_block=512, param=0, staging=0))
+    idx = np.unique(np.concatenate([np.arange(0, batch, 37), np.arange(batch - 200, batch),
+                                    np.arange(0, 64 * 32, 31)]))
+    ref = None
+    for t in ts:
+        out, info, cnt = run_gpu(n, batch, chunk, inter, tune=t)
+        assert np.array_equal(info, np.where(failed, kk + 1, 0)), t
+        assert cnt == int(failed.sum())
+        pads = layout.pad_lane_offsets(n, batch, chunk)
+        assert np.array_equal(out.view(np.uint32)[pads], inter.view(np.uint32)[pads])
+        got = layout.from_interleaved(n, batch, chunk, out)[idx]
+        L64, info64 = oracle.potrf(n, canon[idx])
+        from oracle import checks
+        r = checks.accept(n, canon[idx], got, info[idx], L64, info64)
+        assert r["ok"].all(), (t, np.nonzero(~r["ok"])[0][:5])
+        if ref is None:
+            ref = out
+        else:
+            assert np.array_equal(out.view(np.uint32), ref.view(np.uint32)), t
