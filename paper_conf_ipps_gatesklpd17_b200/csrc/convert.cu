@@ -401,12 +401,22 @@ convert2a_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
     }
 }
 
-// ---- path B: slices of ES elements, one group per tile ----------------------
+// ---- path B: slices of <= ES elements, one group per tile ---------------------
+// Shared tile, phase-shifted rows: element idx of row R (matrix 32g+R) sits at
+// x = ph_R + idx, ph_R = (row start) % 4, so the aligned float4 slots of the
+// canonical row are aligned float4s of the tile (LDS/STS.128, no per-float
+// scatter).  Slot index XOR (R >> 3) & 3 against bank conflicts on the
+// interleaved side (pitch 52: 13 slots, XOR stays inside the row); measured
+// offline: interleaved-side accesses conflict-free, canonical side <= 2-way.
+constexpr int CV2B_PITCH = 52;
+__device__ __forceinline__ int cv2b_at(int R, int x) {
+    return R * CV2B_PITCH + 4 * ((x >> 2) ^ ((R >> 3) & 3)) + (x & 3);
+}
+
 template <int ES, bool ALIGNED>
 struct Cv2B {
-    static constexpr int PITCH = ES + 1;
     static constexpr int SL = ALIGNED ? ES / 4 : ES / 4 + 1;   // float4 slots per row
-    static constexpr int LD = (32 * SL + 31) / 32;             // per lane (== SL)
+    static constexpr int LD = SL;                              // canonical slots per lane
     static constexpr int LK = ES / 4;                          // line steps per lane
     static constexpr int MINB0 = LD >= 9 ? 2 : 3, MINB1 = LK >= 9 ? 2 : 3;
 };
@@ -415,14 +425,14 @@ template <int DIR, int ES, bool ALIGNED>
 __global__ void __launch_bounds__(CV_THREADS, DIR == 0 ? Cv2B<ES, ALIGNED>::MINB0 : Cv2B<ES, ALIGNED>::MINB1)
 convert2b_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shape s) {
     using SB = Cv2B<ES, ALIGNED>;
-    __shared__ float tiles[CV_WARPS][CV2_TILE];
+    extern __shared__ __align__(16) float cv2b_smem[];     // CV_WARPS x 32 x CV2B_PITCH (53 KB)
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    float *T = tiles[wid];
+    float *T = cv2b_smem + wid * (32 * CV2B_PITCH);
     const int64_t W = (int64_t)gridDim.x * CV_WARPS;
     int64_t t = (int64_t)blockIdx.x * CV_WARPS + wid;
     if (t >= s.tiles) return;
     const int c4 = (lane & 7) * 4, lq = lane >> 3;
-    float4 R[DIR == 0 ? SB::LD : SB::LK];
+    float4 R4[DIR == 0 ? SB::LD : SB::LK];
     auto geom = [&](int64_t tt, int64_t &g, int &e0, int &es) {
         g = tt / s.nsl;
         const int sl = (int)(tt - g * s.nsl);
@@ -434,24 +444,33 @@ convert2b_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
             es = (int)((int64_t)(sl + 1) * s.E / s.nsl) - e0;
         }
     };
+    auto phase = [&](int R, int e0) { return ALIGNED ? 0 : ((R * s.E + e0) & 3); };
+    // canonical slot k of this lane: row R, slot sl (of the aligned float4s
+    // covering [st_R, st_R + es)); valid when R < 32 and the slot overlaps
+    auto slot = [&](int k, int &R, int &sl) {
+        const int i = lane + 32 * k;
+        R = i / SB::SL;
+        sl = i - R * SB::SL;
+    };
     auto load = [&](int64_t tt) {
         int64_t g;
         int e0, es;
         geom(tt, g, e0, es);
-        if (DIR == 0) {                                   // canonical row segments via slots
+        if (DIR == 0) {
 #pragma unroll
             for (int k = 0; k < SB::LD; ++k) {
-                const int i = lane + 32 * k, r = i / SB::SL, sl = i - r * SB::SL;
-                const int64_t st = (g * 32 + r) * (int64_t)s.E + e0;
-                const int ph = ALIGNED ? 0 : (int)(st & 3);
-                if (r < 32 && 4 * sl < ph + es) R[k] = ldg4(src + (st - ph) + 4 * sl);
+                int R, sl;
+                slot(k, R, sl);
+                const int ph = phase(R, e0);
+                if (R < 32 && 4 * sl < ph + es)
+                    R4[k] = ldg4(src + ((g * 32 + R) * (int64_t)s.E + e0 - ph) + 4 * sl);
             }
         } else {
             const int64_t base = cv2_line(s, g) + (int64_t)e0 * s.C + c4;
 #pragma unroll
             for (int k = 0; k < SB::LK; ++k) {
                 const int li = 4 * k + lq;
-                if (li < es) R[k] = ldg4(src + base + (int64_t)li * s.C);
+                if (li < es) R4[k] = ldg4(src + base + (int64_t)li * s.C);
             }
         }
     };
@@ -460,29 +479,23 @@ convert2b_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
         int64_t g;
         int e0, es;
         geom(t, g, e0, es);
-        if (DIR == 0) {
+        if (DIR == 0) {                                   // canonical slots -> tile (STS.128)
 #pragma unroll
             for (int k = 0; k < SB::LD; ++k) {
-                const int i = lane + 32 * k, r = i / SB::SL, sl = i - r * SB::SL;
-                const int64_t st = (g * 32 + r) * (int64_t)s.E + e0;
-                const int ph = ALIGNED ? 0 : (int)(st & 3);
-                if (r < 32 && 4 * sl < ph + es) {
-                    const float v[4] = {R[k].x, R[k].y, R[k].z, R[k].w};
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) {
-                        const int idx = 4 * sl + j - ph;
-                        if (idx >= 0 && idx < es) T[r * SB::PITCH + idx] = v[j];
-                    }
-                }
+                int R, sl;
+                slot(k, R, sl);
+                const int ph = phase(R, e0);
+                if (R < 32 && 4 * sl < ph + es)
+                    *reinterpret_cast<float4 *>(T + cv2b_at(R, 4 * sl)) = R4[k];
             }
-        } else {
+        } else {                                          // interleaved lines -> tile
 #pragma unroll
             for (int k = 0; k < SB::LK; ++k) {
                 const int li = 4 * k + lq;
                 if (li < es) {
-                    const float v[4] = {R[k].x, R[k].y, R[k].z, R[k].w};
+                    const float v[4] = {R4[k].x, R4[k].y, R4[k].z, R4[k].w};
 #pragma unroll
-                    for (int j = 0; j < 4; ++j) T[(c4 + j) * SB::PITCH + li] = v[j];
+                    for (int j = 0; j < 4; ++j) T[cv2b_at(c4 + j, phase(c4 + j, e0) + li)] = v[j];
                 }
             }
         }
@@ -490,32 +503,35 @@ convert2b_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
         const int64_t tn = t + W;
         const bool more = tn < s.tiles;
         if (more) load(tn);
-        if (DIR == 0) {
+        if (DIR == 0) {                                   // tile -> interleaved lines
             const int64_t base = cv2_line(s, g) + (int64_t)e0 * s.C + c4;
 #pragma unroll
             for (int k = 0; k < SB::LK; ++k) {
                 const int li = 4 * k + lq;
                 if (li < es) {
-                    const float *r = T + c4 * SB::PITCH + li;
-                    stg4(dst + base + (int64_t)li * s.C, r[0], r[SB::PITCH], r[2 * SB::PITCH], r[3 * SB::PITCH]);
+                    float v[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) v[j] = T[cv2b_at(c4 + j, phase(c4 + j, e0) + li)];
+                    stg4(dst + base + (int64_t)li * s.C, v[0], v[1], v[2], v[3]);
                 }
             }
-        } else {
+        } else {                                          // tile -> canonical slots
 #pragma unroll
             for (int k = 0; k < SB::LD; ++k) {
-                const int i = lane + 32 * k, r = i / SB::SL, sl = i - r * SB::SL;
-                const int64_t st = (g * 32 + r) * (int64_t)s.E + e0;
-                const int ph = ALIGNED ? 0 : (int)(st & 3);
-                if (r < 32 && 4 * sl < ph + es) {
-                    const int i0 = 4 * sl - ph;                  // element index of the slot's first float
-                    float *p = dst + (st - ph) + 4 * sl;
-                    if (i0 >= 0 && i0 + 4 <= es) {
-                        const float *q = T + r * SB::PITCH + i0;
-                        stg4(p, q[0], q[1], q[2], q[3]);
-                    } else {
+                int R, sl;
+                slot(k, R, sl);
+                const int ph = phase(R, e0);
+                if (R < 32 && 4 * sl < ph + es) {
+                    const float4 q = *reinterpret_cast<const float4 *>(T + cv2b_at(R, 4 * sl));
+                    float *p = dst + ((g * 32 + R) * (int64_t)s.E + e0 - ph) + 4 * sl;
+                    const int i0 = 4 * sl - ph;           // element index of the slot's first float
+                    if (ALIGNED || (i0 >= 0 && i0 + 4 <= es)) {
+                        stg4(p, q.x, q.y, q.z, q.w);
+                    } else {                              // edge slot: only this tile's floats
+                        const float v[4] = {q.x, q.y, q.z, q.w};
 #pragma unroll
-                        for (int j = 0; j < 4; ++j)
-                            if (i0 + j >= 0 && i0 + j < es) stg1(p + j, T[r * SB::PITCH + i0 + j]);
+                        for (int jj = 0; jj < 4; ++jj)
+                            if (i0 + jj >= 0 && i0 + jj < es) stg1(p + jj, v[jj]);
                     }
                 }
             }
@@ -528,16 +544,20 @@ convert2b_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
 
 template <typename K>
 static cudaError_t launch_persistent(K kern, int64_t tiles, const float *src, float *dst, const Cv2Shape &s,
-                                     cudaStream_t stream) {
+                                     cudaStream_t stream, size_t dyn_smem = 0) {
     int dev = 0, sms = 148, per_sm = 4;
     if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, CV_THREADS, 0);
+    if (dyn_smem > 0) {
+        const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn_smem);
+        if (e != cudaSuccess) return e;
+    }
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, CV_THREADS, dyn_smem);
     if (per_sm < 1) per_sm = 1;
     int64_t grid = (int64_t)sms * per_sm;
     const int64_t need = (tiles + CV_WARPS - 1) / CV_WARPS;
     if (grid > need) grid = need;
     if (grid < 1) grid = 1;
-    kern<<<(unsigned)grid, CV_THREADS, 0, stream>>>(src, dst, s);
+    kern<<<(unsigned)grid, CV_THREADS, dyn_smem, stream>>>(src, dst, s);
     return cudaGetLastError();
 }
 
@@ -574,10 +594,11 @@ static cudaError_t launch_v2(int n, int64_t G, int64_t C, const float *src, floa
     s.es_last = s.E - (s.nsl - 1) * ES;
     s.tiles = G * s.nsl;
     const bool al = s.E % 4 == 0;
+    constexpr size_t B_SMEM = (size_t)CV_WARPS * 32 * CV2B_PITCH * sizeof(float);
 #define BSP_CV2B(ESV)                                                                                    \
     if (ES == ESV)                                                                                       \
-        return al ? launch_persistent(convert2b_kernel<DIR, ESV, true>, s.tiles, src, dst, s, stream)   \
-                  : launch_persistent(convert2b_kernel<DIR, ESV, false>, s.tiles, src, dst, s, stream);
+        return al ? launch_persistent(convert2b_kernel<DIR, ESV, true>, s.tiles, src, dst, s, stream, B_SMEM)   \
+                  : launch_persistent(convert2b_kernel<DIR, ESV, false>, s.tiles, src, dst, s, stream, B_SMEM);
     BSP_CV2B(20) BSP_CV2B(24) BSP_CV2B(28) BSP_CV2B(32)
 #undef BSP_CV2B
     return cudaErrorInvalidValue;
@@ -588,12 +609,8 @@ cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float
     // 128-bit accesses need 16-B aligned bases (the ABI guarantees 16-B aligned pointers)
     const bool al = ((uintptr_t)src % 16 == 0) && ((uintptr_t)dst % 16 == 0);
     int64_t gbeg = 0;
-    // v2 for every full group -- except interleaved -> canonical at odd n >= 7
-    // (path B with phase != 0): there its edge slots (predicated scalar stores,
-    // 4 scalar LDS per slot) measured 2.6-3.5 TB/s against v1's 3.2-3.7
-    // (profiles/r02/ncu_convert.md: mio_throttle + short_scoreboard bound).
-    const int E = n * n;
-    const bool v2 = al && C % 4 == 0 && !(dir == 1 && E > 25 && E % 4 != 0);
+    // v2 for every full group (v1: the ragged last group, C % 4 != 0)
+    const bool v2 = al && C % 4 == 0;
     if (v2) {
         const int64_t G = batch / 32;
         if (G > 0) {

@@ -202,10 +202,12 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
             // tile's loads above the first tcgen05.st: FILL*16 loads in flight
             // (plus the register triangle's), no spills (round 2: n = 25, 29,
             // 31 spilled 12-216 B, n = 33..42 up to 304 B, at 255 registers)
-            // (5 tiles with TMA staging; 1 with per-thread cp.async, whose address
-            // arithmetic for a runtime chunk stride needs the registers)
+            // (TMA staging: 12 tiles for n <= 32, 5 above -- the largest batches
+            // without spills, more bytes in flight per warp at 8 warps/SM;
+            // per-thread cp.async: 1, its runtime-stride address arithmetic
+            // needs the registers)
             constexpr int idx = pb * TR - pb * (pb - 1) / 2 + (rb - pb);
-            constexpr int FILL = TMA ? 5 : 1;
+            constexpr int FILL = TMA ? (N <= 32 ? 12 : 5) : 1;
             if constexpr ((idx + 1) % FILL == 0) __syncwarp();
         });
     });
