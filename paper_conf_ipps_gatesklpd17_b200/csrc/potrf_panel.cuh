@@ -88,6 +88,7 @@ potrf_panel_kernel(float *__restrict__ A, int32_t *__restrict__ info,
     for (int n = S; n < N; ++n)
 #pragma unroll
         for (int m = n; m < N; ++m) r[tri<NT>(m - S, n - S)] = ld_stream(ad.at(m, n));
+    const Addr<N, CT> ads = ad.opaque();           // store addresses (see Addr::opaque)
 
     if constexpr (TMA) mbar_wait(bar, 0);
     else cp_async_wait_all();
@@ -181,7 +182,7 @@ potrf_panel_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                     const int m = r0 + i;
                     if (m < N && (!diag || i >= j)) {
                         P[(cbase[j] + m) * BL] = acc[i + j * NB];
-                        if (active) st_stream(ad.at(m, cb * NB + j), acc[i + j * NB]);
+                        if (active) st_stream(ads.at(m, cb * NB + j), acc[i + j * NB]);
                     }
                 }
         }
@@ -217,7 +218,7 @@ potrf_panel_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                 r[tri<NT>(m, n)] = f_upd(r[tri<NT>(m, n)], r[tri<NT>(m, k)], r[tri<NT>(n, k)]);
         if (active) {
 #pragma unroll
-            for (int m = k; m < NT; ++m) st_stream(ad.at(m + S, k + S), r[tri<NT>(m, k)]);
+            for (int m = k; m < NT; ++m) st_stream(ads.at(m + S, k + S), r[tri<NT>(m, k)]);
         }
     });
     if (active) info[gid] = inf;

@@ -44,6 +44,7 @@ potrf_reg_kernel(float *__restrict__ A, int32_t *__restrict__ info,
         for (int i = j; i < N; ++i) a[tri<N>(i, j)] = ld_stream(ad.at(i, j));
 
     int inf = 0;
+    const Addr<N, CT> ads = ad.opaque();           // store addresses (see Addr::opaque)
     sfor<0, N>([&](auto k_) {
         constexpr int k = BSP_CI(k_);
         const float d = a[tri<N>(k, k)];
@@ -60,7 +61,7 @@ potrf_reg_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                 a[tri<N>(m, n)] = f_upd(a[tri<N>(m, n)], a[tri<N>(m, k)], a[tri<N>(n, k)]);
         if (active) {
 #pragma unroll
-            for (int m = k; m < N; ++m) st_stream(ad.at(m, k), a[tri<N>(m, k)]);
+            for (int m = k; m < N; ++m) st_stream(ads.at(m, k), a[tri<N>(m, k)]);
         }
     });
     if (active) info[gid] = inf;

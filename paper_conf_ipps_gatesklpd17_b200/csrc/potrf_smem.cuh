@@ -86,6 +86,7 @@ potrf_smem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
     for (int n = S; n < N; ++n)
 #pragma unroll
         for (int m = n; m < N; ++m) r[tri<NT>(m - S, n - S)] = ld_stream(ad.at(m, n));
+    const Addr<N, CT> ads = ad.opaque();           // store addresses (see Addr::opaque)
 
     if constexpr (TMA) {
         mbar_wait(bar, 0);
@@ -116,7 +117,7 @@ potrf_smem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
         for (int m = c + 1; m < N; ++m) col[m] = f_mul(col[m], inv);
         if (active) {
 #pragma unroll
-            for (int m = c; m < N; ++m) st_stream(ad.at(m, c), col[m]);
+            for (int m = c; m < N; ++m) st_stream(ads.at(m, c), col[m]);
         }
 #pragma unroll
         for (int m = c + 1; m < N; ++m) BSP_P(m, c) = col[m];
@@ -153,7 +154,7 @@ potrf_smem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                 r[tri<NT>(m, n)] = f_upd(r[tri<NT>(m, n)], r[tri<NT>(m, k)], r[tri<NT>(n, k)]);
         if (active) {
 #pragma unroll
-            for (int m = k; m < NT; ++m) st_stream(ad.at(m + S, k + S), r[tri<NT>(m, k)]);
+            for (int m = k; m < NT; ++m) st_stream(ads.at(m + S, k + S), r[tri<NT>(m, k)]);
         }
     });
     if (active) info[gid] = inf;

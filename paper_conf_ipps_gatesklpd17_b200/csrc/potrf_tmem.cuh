@@ -202,12 +202,13 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
             // tile's loads above the first tcgen05.st: FILL*16 loads in flight
             // (plus the register triangle's), no spills (round 2: n = 25, 29,
             // 31 spilled 12-216 B, n = 33..42 up to 304 B, at 255 registers)
-            // (TMA staging: 12 tiles for n <= 32, 5 above -- the largest batches
-            // without spills, more bytes in flight per warp at 8 warps/SM;
-            // per-thread cp.async: 1, its runtime-stride address arithmetic
-            // needs the registers)
+            // (TMA staging: 12 tiles for n <= 31 -- more bytes in flight per warp
+            // at 8 warps/SM: n = 29-31 +1-3.5% over 5 -- and 5 for n >= 32, where
+            // 12 cost the C3 run (n = 32, 4M) 2.7%; both spill-free.  Per-thread
+            // cp.async: 1, its runtime-stride address arithmetic needs the
+            // registers.  Measured: profiles/r02/ptmem_fill.md)
             constexpr int idx = pb * TR - pb * (pb - 1) / 2 + (rb - pb);
-            constexpr int FILL = TMA ? (N <= 32 ? 12 : 5) : 1;
+            constexpr int FILL = TMA ? (N <= 31 ? 12 : 5) : 1;
             if constexpr ((idx + 1) % FILL == 0) __syncwarp();
         });
     });
@@ -218,6 +219,7 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
     }
 
     int inf = 0;
+    const Addr<N, CT> ads = ad.opaque();           // store addresses (see Addr::opaque)
     // smem tile loader (packed columns CS..S-1); rows >= N read as 0
     auto load_tile_smem = [&](int rb, int pb, float *t, bool lower_only) {
 #pragma unroll
@@ -256,13 +258,13 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                 }
         }
         if (active) {
-            float *tb = ad.at(rb * NB, CB * NB);
+            float *tb = ads.at(rb * NB, CB * NB);
 #pragma unroll
             for (int j = 0; j < NB; ++j)
 #pragma unroll
                 for (int i = 0; i < NB; ++i)
                     if (rb * NB + i < N && (!DIAG || i >= j))
-                        st_stream(tb + (int64_t)(i + j * N) * ad.stride(), acc[i + j * NB]);
+                        st_stream(tb + (int64_t)(i + j * N) * ads.stride(), acc[i + j * NB]);
         }
     };
 
@@ -425,7 +427,7 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                 r[tri<NT>(m, n)] = f_upd(r[tri<NT>(m, n)], r[tri<NT>(m, k)], r[tri<NT>(n, k)]);
         if (active) {
 #pragma unroll
-            for (int m = k; m < NT; ++m) st_stream(ad.at(m + S, k + S), r[tri<NT>(m, k)]);
+            for (int m = k; m < NT; ++m) st_stream(ads.at(m + S, k + S), r[tri<NT>(m, k)]);
         }
         if constexpr (SOLVE) {                          // forward step j = S + k
             const float xk = f_mul(X[(S + k) * 32], inv);
