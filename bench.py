@@ -561,7 +561,7 @@ def run_ours(a, w):
         per_n = per_n_sweep(bsp, torch, dev, stream, ns, 1 << 20, 32, peak=peak, tag="1M")
         small_ns = [x for x in ns if x <= 4]
         if small_ns:
-            per_n_large = per_n_sweep(bsp, torch, dev, stream, small_ns, 1 << 26, 32, conv=False,
+            per_n_large = per_n_sweep(bsp, torch, dev, stream, small_ns, 1 << 26, 32, conv=True,
                                       peak=peak, tag="64M (n <= 4 leave the launch-latency regime)")
 
     cpu = None

@@ -75,8 +75,10 @@ enum {
     BSPOTRF_VARIANT_PTMEM = 5, /* PANEL with the first panel tile columns held in
                                  Tensor Memory (tcgen05.ld/st), 128-thread
                                  CTAs with 256 TMEM columns each (two per SM;
-                                 512, one per SM, for n > 32); TMA staging
-                                 needs chunk 32; 24 <= n <= 44               */
+                                 512, one per SM, for n > 32); staging 1 =
+                                 TMA (chunk 32), TMEM fill in batches of 5
+                                 tiles; 3 = TMA, batches of 12 (n <= 32);
+                                 2 = per-thread cp.async; 24 <= n <= 44       */
     BSPOTRF_VARIANT_RTMA = 6, /* REG with TMA bulk copies in and out of a
                                  shared-memory image (chunk 32 only); `param`
                                  warps per CTA (2 or 4); 4 <= n <= 20         */

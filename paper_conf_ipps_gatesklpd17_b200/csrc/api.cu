@@ -112,7 +112,9 @@ static LaunchFn resolve(int n, int chunk, const bspotrf_tuning &t, int *tpb_out)
     case BSPOTRF_VARIANT_PTMEM: {
         int staging = t.staging == 0 ? (chunk == 32 ? 1 : 2) : t.staging;
         *tpb_out = 128;
-        if (staging == 1) return chunk == 32 ? find(BSPOTRF_VARIANT_PTMEM, n, t.param, 32, 1) : nullptr;
+        // 1: TMA, fill batches of 5 tiles; 3: TMA, batches of 12 (instance tma = 3)
+        if (staging == 1 || staging == 3)
+            return chunk == 32 ? find(BSPOTRF_VARIANT_PTMEM, n, t.param, 32, staging) : nullptr;
         LaunchFn f = find(BSPOTRF_VARIANT_PTMEM, n, t.param, chunk == 32 ? 32 : 0, 0);
         return f ? f : find(BSPOTRF_VARIANT_PTMEM, n, t.param, 0, 0);
     }

@@ -418,7 +418,7 @@ struct Cv2B {
     static constexpr int SL = ALIGNED ? ES / 4 : ES / 4 + 1;   // float4 slots per row
     static constexpr int LD = SL;                              // canonical slots per lane
     static constexpr int LK = ES / 4;                          // line steps per lane
-    static constexpr int MINB0 = LD >= 9 ? 2 : 3, MINB1 = LK >= 9 ? 2 : 3;
+    static constexpr int MINB0 = 2, MINB1 = 2;   // 128 registers: per-lane slot tables + 9 float4s
 };
 
 template <int DIR, int ES, bool ALIGNED>
@@ -432,6 +432,35 @@ convert2b_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
     int64_t t = (int64_t)blockIdx.x * CV_WARPS + wid;
     if (t >= s.tiles) return;
     const int c4 = (lane & 7) * 4, lq = lane >> 3;
+    // Per-lane constants, hoisted out of the tile loop (the index arithmetic was
+    // the bound: IMAD/LOP3/BRA ~52% of issue samples at n = 63, round 2):
+    //  canonical slot k: row R, slot sl -> shared offset, row-start phase part
+    //  (R*E mod 4) and the float offset R*E + 4*sl inside the group's block;
+    //  interleaved side: rows c4 + j share the XOR key (c4 >> 3) & 3.
+    // meta[k] = sl | (R*E mod 4) << 8, or -1 for a slot past row 31
+    int soff[SB::LD], rowoff[SB::LD], meta[SB::LD];
+#pragma unroll
+    for (int k = 0; k < SB::LD; ++k) {
+        const int i = lane + 32 * k, R = i / SB::SL, sl = i - R * SB::SL;
+        const int Rc = R < 32 ? R : 0;
+        soff[k] = cv2b_at(Rc, 4 * sl);
+        rowoff[k] = Rc * s.E + 4 * sl;
+        meta[k] = R < 32 ? (sl | (((Rc * s.E) & 3) << 8)) : -1;
+    }
+    auto slot_ok = [&](int k, int ph, int es) { return meta[k] >= 0 && 4 * (meta[k] & 0xff) < ph + es; };
+    auto slot_ph = [&](int k, int e0) { return ALIGNED ? 0 : (((meta[k] >> 8) + e0) & 3); };
+    const int key = (c4 >> 3) & 3;
+    int jbase[4], jph[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        jbase[j] = (c4 + j) * CV2B_PITCH;
+        jph[j] = ((c4 + j) * s.E) & 3;
+    }
+    // interleaved element li = 4k + lq of row c4 + j at x = ph_j + li
+    auto iaddr = [&](int j, int k, int ph) {
+        const int u = ph + lq;                            // 0..6
+        return jbase[j] + (u & 3) + 4 * (((u >> 2) + k) ^ key);
+    };
     float4 R4[DIR == 0 ? SB::LD : SB::LK];
     auto geom = [&](int64_t tt, int64_t &g, int &e0, int &es) {
         g = tt / s.nsl;
@@ -444,33 +473,23 @@ convert2b_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
             es = (int)((int64_t)(sl + 1) * s.E / s.nsl) - e0;
         }
     };
-    auto phase = [&](int R, int e0) { return ALIGNED ? 0 : ((R * s.E + e0) & 3); };
-    // canonical slot k of this lane: row R, slot sl (of the aligned float4s
-    // covering [st_R, st_R + es)); valid when R < 32 and the slot overlaps
-    auto slot = [&](int k, int &R, int &sl) {
-        const int i = lane + 32 * k;
-        R = i / SB::SL;
-        sl = i - R * SB::SL;
-    };
     auto load = [&](int64_t tt) {
         int64_t g;
         int e0, es;
         geom(tt, g, e0, es);
-        if (DIR == 0) {
+        if (DIR == 0) {                                   // canonical slots
+            const float *gb = src + g * 32 * (int64_t)s.E + e0;
 #pragma unroll
             for (int k = 0; k < SB::LD; ++k) {
-                int R, sl;
-                slot(k, R, sl);
-                const int ph = phase(R, e0);
-                if (R < 32 && 4 * sl < ph + es)
-                    R4[k] = ldg4(src + ((g * 32 + R) * (int64_t)s.E + e0 - ph) + 4 * sl);
+                const int ph = slot_ph(k, e0);
+                if (slot_ok(k, ph, es)) R4[k] = ldg4(gb + rowoff[k] - ph);
             }
-        } else {
-            const int64_t base = cv2_line(s, g) + (int64_t)e0 * s.C + c4;
+        } else {                                          // interleaved lines
+            const float *lb = src + cv2_line(s, g) + (int64_t)e0 * s.C + c4;
 #pragma unroll
             for (int k = 0; k < SB::LK; ++k) {
                 const int li = 4 * k + lq;
-                if (li < es) R4[k] = ldg4(src + base + (int64_t)li * s.C);
+                if (li < es) R4[k] = ldg4(lb + (int64_t)li * s.C);
             }
         }
     };
@@ -479,23 +498,22 @@ convert2b_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
         int64_t g;
         int e0, es;
         geom(t, g, e0, es);
+        int ph4[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) ph4[j] = ALIGNED ? 0 : ((jph[j] + e0) & 3);
         if (DIR == 0) {                                   // canonical slots -> tile (STS.128)
 #pragma unroll
             for (int k = 0; k < SB::LD; ++k) {
-                int R, sl;
-                slot(k, R, sl);
-                const int ph = phase(R, e0);
-                if (R < 32 && 4 * sl < ph + es)
-                    *reinterpret_cast<float4 *>(T + cv2b_at(R, 4 * sl)) = R4[k];
+                const int ph = slot_ph(k, e0);
+                if (slot_ok(k, ph, es)) *reinterpret_cast<float4 *>(T + soff[k]) = R4[k];
             }
         } else {                                          // interleaved lines -> tile
 #pragma unroll
             for (int k = 0; k < SB::LK; ++k) {
-                const int li = 4 * k + lq;
-                if (li < es) {
+                if (4 * k + lq < es) {
                     const float v[4] = {R4[k].x, R4[k].y, R4[k].z, R4[k].w};
 #pragma unroll
-                    for (int j = 0; j < 4; ++j) T[cv2b_at(c4 + j, phase(c4 + j, e0) + li)] = v[j];
+                    for (int j = 0; j < 4; ++j) T[iaddr(j, k, ph4[j])] = v[j];
                 }
             }
         }
@@ -504,27 +522,26 @@ convert2b_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
         const bool more = tn < s.tiles;
         if (more) load(tn);
         if (DIR == 0) {                                   // tile -> interleaved lines
-            const int64_t base = cv2_line(s, g) + (int64_t)e0 * s.C + c4;
+            float *lb = dst + cv2_line(s, g) + (int64_t)e0 * s.C + c4;
 #pragma unroll
             for (int k = 0; k < SB::LK; ++k) {
                 const int li = 4 * k + lq;
                 if (li < es) {
                     float v[4];
 #pragma unroll
-                    for (int j = 0; j < 4; ++j) v[j] = T[cv2b_at(c4 + j, phase(c4 + j, e0) + li)];
-                    stg4(dst + base + (int64_t)li * s.C, v[0], v[1], v[2], v[3]);
+                    for (int j = 0; j < 4; ++j) v[j] = T[iaddr(j, k, ph4[j])];
+                    stg4(lb + (int64_t)li * s.C, v[0], v[1], v[2], v[3]);
                 }
             }
         } else {                                          // tile -> canonical slots
+            float *gb = dst + g * 32 * (int64_t)s.E + e0;
 #pragma unroll
             for (int k = 0; k < SB::LD; ++k) {
-                int R, sl;
-                slot(k, R, sl);
-                const int ph = phase(R, e0);
-                if (R < 32 && 4 * sl < ph + es) {
-                    const float4 q = *reinterpret_cast<const float4 *>(T + cv2b_at(R, 4 * sl));
-                    float *p = dst + ((g * 32 + R) * (int64_t)s.E + e0 - ph) + 4 * sl;
-                    const int i0 = 4 * sl - ph;           // element index of the slot's first float
+                const int ph = slot_ph(k, e0);
+                if (slot_ok(k, ph, es)) {
+                    const float4 q = *reinterpret_cast<const float4 *>(T + soff[k]);
+                    float *p = gb + rowoff[k] - ph;
+                    const int i0 = 4 * (meta[k] & 0xff) - ph;   // element index of the slot's first float
                     if (ALIGNED || (i0 >= 0 && i0 + 4 <= es)) {
                         stg4(p, q.x, q.y, q.z, q.w);
                     } else {                              // edge slot: only this tile's floats

@@ -51,7 +51,7 @@ cudaError_t launch_panel(const FactorArgs &a);
 
 // Variant PTMEM: PANEL with the first panel tile columns in Tensor Memory
 // (csrc/potrf_tmem.cuh); 4-warp CTAs, 256 TMEM columns each.
-template <int N, int CT, int S, bool TMA>
+template <int N, int CT, int S, bool TMA, int FILL = 0>
 cudaError_t launch_ptmem(const FactorArgs &a);
 
 // Variant RTMA: REG with TMA bulk staging in and out (chunk 32 only), W warps

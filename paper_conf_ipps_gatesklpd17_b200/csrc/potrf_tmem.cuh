@@ -105,7 +105,10 @@ struct TmemShape {
 // register tail, backward substitution reads L back from TMEM / shared memory /
 // registers.  x lives in shared memory ([i][lane], after the panel part).  Op
 // order is potrs.cuh's, so X is bitwise identical to factor-then-SPOTRS.
-template <int N, int CT, int S, bool TMA, bool SOLVE = false>
+// FILLT: TMEM tiles loaded per warp-synchronised batch of the fill (0 = the
+// default: 5 with TMA staging, 1 with per-thread cp.async); a tuning axis
+// (bspotrf_tuning.staging 3 = TMA with 12), see the fill below.
+template <int N, int CT, int S, bool TMA, bool SOLVE = false, int FILLT = 0>
 __global__ void __launch_bounds__(128, TmemShape<N, S>::COLS == 256 ? 2 : 1)
 potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                    int32_t *__restrict__ nfailed, int64_t batch, int64_t cs,
@@ -202,13 +205,13 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
             // tile's loads above the first tcgen05.st: FILL*16 loads in flight
             // (plus the register triangle's), no spills (round 2: n = 25, 29,
             // 31 spilled 12-216 B, n = 33..42 up to 304 B, at 255 registers)
-            // (TMA staging: 12 tiles for n <= 31 -- more bytes in flight per warp
-            // at 8 warps/SM: n = 29-31 +1-3.5% over 5 -- and 5 for n >= 32, where
-            // 12 cost the C3 run (n = 32, 4M) 2.7%; both spill-free.  Per-thread
-            // cp.async: 1, its runtime-stride address arithmetic needs the
-            // registers.  Measured: profiles/r02/ptmem_fill.md)
+            // (TMA staging: 5 tiles, or 12 as the FILLT tuning axis -- more bytes
+            // in flight per warp at 8 warps/SM: n = 29-31 +1-3.5%, n = 26/28 -7%:
+            // the table picks per n, profiles/r02/ptmem_fill.md; both spill-free.
+            // Per-thread cp.async: 1, its runtime-stride address arithmetic
+            // needs the registers.)
             constexpr int idx = pb * TR - pb * (pb - 1) / 2 + (rb - pb);
-            constexpr int FILL = TMA ? (N <= 31 ? 12 : 5) : 1;
+            constexpr int FILL = FILLT ? FILLT : (TMA ? 5 : 1);
             if constexpr ((idx + 1) % FILL == 0) __syncwarp();
         });
     });
@@ -491,7 +494,7 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
     }
 }
 
-template <int N, int CT, int S, bool TMA>
+template <int N, int CT, int S, bool TMA, int FILL>
 cudaError_t launch_ptmem(const FactorArgs &a) {
     using SH = TmemShape<N, S>;
     // Enough dynamic shared memory that at most 512 / COLS CTAs are resident
@@ -500,7 +503,7 @@ cudaError_t launch_ptmem(const FactorArgs &a) {
     size_t sm = (size_t)4 * SH::PSM * 32 * 4;
     const size_t floor_sm = SH::COLS == 256 ? 80 * 1024 : 120 * 1024;
     if (sm < floor_sm) sm = floor_sm;
-    auto kern = potrf_ptmem_kernel<N, CT, S, TMA, false>;
+    auto kern = potrf_ptmem_kernel<N, CT, S, TMA, false, FILL>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e == cudaSuccess) e = apply_carveout(kern, a.carveout);
     if (e != cudaSuccess) return e;

@@ -87,6 +87,8 @@ def candidates(n, chunk):
         for s in gen_instances.ptmem_s_values(n):
             if chunk == 32:
                 c.append(dict(variant=PTMEM, threads_per_block=128, param=s, staging=1))
+                if n <= 32:
+                    c.append(dict(variant=PTMEM, threads_per_block=128, param=s, staging=3))
             c.append(dict(variant=PTMEM, threads_per_block=128, param=s, staging=2))
     if 17 <= n <= 32:
         for s in (n - 16, n - 14, n - 12):

@@ -73,6 +73,8 @@ def main():
             tma = 1 if e["staging"] == 1 or (e["staging"] == 0 and (c == 32 if v == 5 else tmpl)) else 0
             ct = c if tma else (32 if c == 32 else 0)
             want = [n, ct, e["param"], tma] + ([0] if v == 5 else [])
+            if v == 5 and e["staging"] == 3:          # TMA, fill batches of 12 (FILLT template arg)
+                want = [n, 32, e["param"], 1, 0, 12]
         elif v in (10,):
             want = [n, 32 if c == 32 else 0, e["param"]]
         elif v == 12:

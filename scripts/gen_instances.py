@@ -277,6 +277,9 @@ def main():
                 t = "true" if tma else "false"
                 body.append(f"template cudaError_t launch_ptmem<{n}, {ct}, {s}, {t}>(const FactorArgs &);")
                 entries.append(f"{{5, {n}, {s}, {ct}, {int(tma)}, &launch_ptmem<{n}, {ct}, {s}, {t}>}}")
+                if tma and n <= 32:                   # fill-batch axis: staging 3 = TMA, 12 tiles
+                    body.append(f"template cudaError_t launch_ptmem<{n}, {ct}, {s}, true, 12>(const FactorArgs &);")
+                    entries.append(f"{{5, {n}, {s}, {ct}, 3, &launch_ptmem<{n}, {ct}, {s}, true, 12>}}")
                 if sposv_ptmem_fits(n, s):
                     body.append(f"template cudaError_t launch_sposv_ptmem<{n}, {ct}, {s}, {t}>(const SolveArgs &);")
                     sposv_ptmem_entries.append(

@@ -203,6 +203,7 @@ def _tunings(n, chunk):
             out.append(dict(variant=bsp.VARIANT_PTMEM, threads_per_block=128, param=s, staging=2))
             if chunk == 32:
                 out.append(dict(variant=bsp.VARIANT_PTMEM, threads_per_block=128, param=s, staging=1))
+                out.append(dict(variant=bsp.VARIANT_PTMEM, threads_per_block=128, param=s, staging=3))
     for m, fast in gen_instances_mod().regx_combos(n) if n in gen_instances_mod().REGX_N else []:
         if not fast:                              # IEEE: same op sequence -> same bits
             out.append(dict(variant=bsp.VARIANT_REGX, threads_per_block=128, param=m, staging=0))
