@@ -100,6 +100,19 @@ potrf_rcw16_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *_
                                  (uint32_t)((N - j) * 128), &mbar[half]);
                 }
             }
+        } else if (g * 32 + 31 < batch && cs % 4 == 0) {
+            // full group: 16-B copies, 8 lanes per 128-B line (as RCW)
+            const float *gb = A + ((g * 32) / cs) * cs * (int64_t)(N * N) + (g * 32) % cs;
+            const int l8 = q & 7, sub = q >> 3;
+#pragma unroll
+            for (int tt = 0; tt < 2 * RS; ++tt) {
+                const int idx = 4 * tt + sub, r = idx >> 3, w = idx & 7;
+                const int i = P * r + h;
+                if (i >= 8 * c && i < N && 8 * c + w < N && 8 * c + w <= i)
+                    cp_async16(stg + (w * SH::rs(c) + i - 8 * c) * 32 + 4 * l8,
+                               gb + (int64_t)(i + (8 * c + w) * N) * cs + 4 * l8);
+            }
+            cp_async_commit();
         } else {
             const int64_t gm = g * 32 + q;
             const Addr<N, CT> ad(A, gm < batch ? gm : batch - 1, cs);

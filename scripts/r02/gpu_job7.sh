@@ -15,8 +15,8 @@ smoke)
   timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "smoke rc=$?" >> $O/smoke.log
   tail -n 4 $O/smoke.log ;;
 bench)
-  /usr/bin/time -v timeout 900 python bench.py --steps 20 --warmup 5 > $O/bench.json 2> $O/bench.err; echo "bench rc=$?"
-  grep -E "Elapsed|Maximum resident" $O/bench.err ;;
+  t0=$(date +%s); timeout 900 python bench.py --steps 20 --warmup 5 > $O/bench.json 2> $O/bench.err; echo "bench rc=$? wall=$(( $(date +%s) - t0 ))s"
+  tail -c 400 $O/bench.err ;;
 ref)
   timeout 600 python bench.py --impl reference --steps 20 --warmup 5 > $O/bench_ref.json 2> $O/bench_ref.err; echo "ref rc=$?" ;;
 launches)
