@@ -111,11 +111,16 @@ enum {
                                  needs C % 4 == 0 (C = chunk, or batch when
                                  chunk == 0), else runs REG (same bits);
                                  <= 128 threads per block; 1 <= n <= 8        */
-    BSPOTRF_VARIANT_RCW16 = 12 /* RCW with 16 warps per 32 matrices (rows
+    BSPOTRF_VARIANT_RCW16 = 12,/* RCW with 16 warps per 32 matrices (rows
                                  16r+h), one CTA per SM; faster than RCW where
                                  the input comes by per-thread copies (chunk
                                  != 32), slower with chunk 32 (TMA path);
                                  any chunk; 49 <= n <= 64                     */
+    BSPOTRF_VARIANT_RCWD = 13  /* RCW plus a ninth warp that factors each 8x8
+                                 diagonal block while the row warps run the
+                                 GEMM of their other rows (two passes over the
+                                 row buffer); one CTA per SM; any chunk;
+                                 49 <= n <= 64                                */
 };
 
 /* Launch tuning (a row of the autotuning table). */

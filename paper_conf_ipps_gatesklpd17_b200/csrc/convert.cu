@@ -559,6 +559,130 @@ convert2b_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
     }
 }
 
+// ---- interleaved -> canonical at odd n (E % 4 != 0): row streams with carries
+// In path B the two partial float4 slots of every row segment (unaligned slice
+// edges) were stored as scalars, half-sector writes shared with the tile of the
+// neighbouring slice (2.6-3.5 TB/s).  Here one warp runs ALL slices of a group
+// in order, so a row's canonical output is one stream: the partial last slot of
+// a slice stays in the shared tile (copied to the row's front) and completes the
+// first slot of the next slice; the partial first slot of a row (it shares a
+// float4 with the previous row's end) is kept in H and stored with that row's
+// last slot.  Every store is a full, aligned STG.128.
+constexpr int CV2D_WARP = 32 * CV2B_PITCH + 32 * 4;      // tile + per-row head buffer H
+
+template <int ES>
+__global__ void __launch_bounds__(CV_THREADS, 2)
+convert2d_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shape s) {
+    constexpr int SL = ES / 4 + 1;                       // float4 slots per row segment (phase <= 3)
+    constexpr int LK = ES / 4;
+    extern __shared__ __align__(16) float cv2d_smem[];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    float *T = cv2d_smem + wid * CV2D_WARP;
+    float *H = T + 32 * CV2B_PITCH;                      // H[R*4 + j]: head floats of row R
+    const int64_t W = (int64_t)gridDim.x * CV_WARPS;
+    int64_t g = (int64_t)blockIdx.x * CV_WARPS + wid;
+    if (g >= s.G) return;
+    const int c4 = (lane & 7) * 4, lq = lane >> 3;
+    const int key = (c4 >> 3) & 3;
+    auto slice = [&](int sl, int &e0, int &es) {
+        e0 = (int)((int64_t)sl * s.E / s.nsl);
+        es = (int)((int64_t)(sl + 1) * s.E / s.nsl) - e0;
+    };
+    auto iaddr = [&](int R, int x) { return R * CV2B_PITCH + 4 * ((x >> 2) ^ key) + (x & 3); };
+    float4 R4[LK];
+    auto load = [&](int64_t gg, int sl) {
+        int e0, es;
+        slice(sl, e0, es);
+        const float *lb = src + cv2_line(s, gg) + (int64_t)e0 * s.C + c4;
+#pragma unroll
+        for (int k = 0; k < LK; ++k) {
+            const int li = 4 * k + lq;
+            if (li < es) R4[k] = ldg4(lb + (int64_t)li * s.C);
+        }
+    };
+    int sl = 0;
+    load(g, 0);
+    for (;;) {
+        int e0, es;
+        slice(sl, e0, es);
+        const bool first = sl == 0, last = sl == s.nsl - 1;
+        // interleaved lines -> tile rows at x = ph_R + li (ph_R = carry length)
+#pragma unroll
+        for (int k = 0; k < LK; ++k) {
+            const int li = 4 * k + lq;
+            if (li < es) {
+                const float v[4] = {R4[k].x, R4[k].y, R4[k].z, R4[k].w};
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const int R = c4 + j;
+                    T[iaddr(R, (((R * s.E + e0) & 3) + li))] = v[j];
+                }
+            }
+        }
+        __syncwarp();
+        // next slice's (or group's) loads in flight during the stores
+        int64_t gn = g;
+        int sln = sl + 1;
+        if (last) {
+            gn = g + W;
+            sln = 0;
+        }
+        const bool more = gn < s.G;
+        if (more) load(gn, sln);
+        // full slots of every row; the first slot of a row's first slice is its
+        // head (-> H), the partial last slot is the carry (stays) -- except at
+        // the last slice, where it is completed by the next row's head
+        float *gb = dst + g * 32 * (int64_t)s.E;
+#pragma unroll
+        for (int k = 0; k < SL; ++k) {
+            const int i = lane + 32 * k, R = i / SL, sl4 = i - R * SL;
+            if (R < 32) {
+                const int ph = (R * s.E + e0) & 3;
+                const int end = ph + es;                  // floats of the row in the tile
+                const int64_t a0 = (int64_t)R * s.E + e0 - ph;   // stream position of x = 0
+                if (4 * sl4 + 4 <= end) {
+                    const float *t4 = T + R * CV2B_PITCH + 4 * (sl4 ^ ((R >> 3) & 3));
+                    if (first && sl4 == 0 && ph != 0) {
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) H[R * 4 + j] = t4[j];   // head (j >= ph valid)
+                    } else {
+                        stg4(gb + a0 + 4 * sl4, t4[0], t4[1], t4[2], t4[3]);
+                    }
+                } else if (last && 4 * sl4 < end && R < 31) {
+                    // tail (end % 4 floats) + the next row's head = one aligned float4
+                    const int rem = end & 3;
+                    const float *t4 = T + R * CV2B_PITCH + 4 * (sl4 ^ ((R >> 3) & 3));
+                    float v[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) v[j] = j < rem ? t4[j] : H[(R + 1) * 4 + j];
+                    stg4(gb + a0 + 4 * sl4, v[0], v[1], v[2], v[3]);
+                }
+            }
+        }
+        if (!more) break;
+        __syncwarp();
+        if (!last) {
+            // carry: the row's partial last slot moves to the row's front (slot 0)
+            // -- the next slice puts its data after it (its phase == the carry length)
+            const int R = lane;
+            const int end = ((R * s.E + e0) & 3) + es, rem = end & 3;
+            if (rem) {
+                const float *t4 = T + R * CV2B_PITCH + 4 * (((end >> 2)) ^ ((R >> 3) & 3));
+                float *f4 = T + R * CV2B_PITCH + 4 * (0 ^ ((R >> 3) & 3));
+                float v[3];
+#pragma unroll
+                for (int j = 0; j < 3; ++j) v[j] = t4[j];
+#pragma unroll
+                for (int j = 0; j < 3; ++j)
+                    if (j < rem) f4[j] = v[j];
+            }
+            __syncwarp();
+        }
+        g = gn;
+        sl = sln;
+    }
+}
+
 template <typename K>
 static cudaError_t launch_persistent(K kern, int64_t tiles, const float *src, float *dst, const Cv2Shape &s,
                                      cudaStream_t stream, size_t dyn_smem = 0) {
@@ -612,6 +736,13 @@ static cudaError_t launch_v2(int n, int64_t G, int64_t C, const float *src, floa
     s.tiles = G * s.nsl;
     const bool al = s.E % 4 == 0;
     constexpr size_t B_SMEM = (size_t)CV_WARPS * 32 * CV2B_PITCH * sizeof(float);
+    constexpr size_t D_SMEM = (size_t)CV_WARPS * CV2D_WARP * sizeof(float);
+    if (DIR == 1 && !al) {                                // row streams: a warp per group
+#define BSP_CV2D(ESV) \
+    if (ES == ESV) return launch_persistent(convert2d_kernel<ESV>, G, src, dst, s, stream, D_SMEM);
+        BSP_CV2D(20) BSP_CV2D(24) BSP_CV2D(28) BSP_CV2D(32)
+#undef BSP_CV2D
+    }
 #define BSP_CV2B(ESV)                                                                                    \
     if (ES == ESV)                                                                                       \
         return al ? launch_persistent(convert2b_kernel<DIR, ESV, true>, s.tiles, src, dst, s, stream, B_SMEM)   \
@@ -623,6 +754,9 @@ static cudaError_t launch_v2(int n, int64_t G, int64_t C, const float *src, floa
 
 cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float *src, float *dst,
                            cudaStream_t stream) {
+    // n = 1: element (0,0) of matrix b sits at offset b in BOTH layouts
+    // ((b/C)*C + b%C = b; pad lanes only follow the last real matrix): a copy
+    if (n == 1) return cudaMemcpyAsync(dst, src, (size_t)batch * sizeof(float), cudaMemcpyDeviceToDevice, stream);
     // 128-bit accesses need 16-B aligned bases (the ABI guarantees 16-B aligned pointers)
     const bool al = ((uintptr_t)src % 16 == 0) && ((uintptr_t)dst % 16 == 0);
     int64_t gbeg = 0;

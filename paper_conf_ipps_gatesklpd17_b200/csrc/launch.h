@@ -90,6 +90,10 @@ cudaError_t launch_regv(const FactorArgs &a);
 template <int N, int CT>
 cudaError_t launch_rcw16(const FactorArgs &a);
 
+// Variant RCWD: RCW with a diagonal-factorization warp (csrc/potrf_rcwd.cuh).
+template <int N, int CT>
+cudaError_t launch_rcwd(const FactorArgs &a);
+
 // Variant TILE: the paper's top-looking tile algorithm, NB x NB register
 // tiles streamed from global memory, runtime chunk stride (csrc/potrf_tile.cuh).
 template <int N, int NB>

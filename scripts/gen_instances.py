@@ -52,6 +52,7 @@ QTM_CT = (32, 0)
 REGV_N = range(1, 9)
 RCW_N = range(33, 65)
 RCW16_N = range(49, 65)
+RCWD_N = range(49, 65)
 RCW_CT = (32, 0)
 
 
@@ -319,6 +320,15 @@ def main():
             entries.append(f"{{12, {n}, 0, {ct}, 0, &launch_rcw16<{n}, {ct}>}}")
         body.append("}  // namespace bsp\n")
         name = f"inst_rcw16_{n:02d}.cu"
+        write_if_changed(os.path.join(GEN, name), "\n".join(body))
+        files.add(name)
+    for n in RCWD_N:
+        body = [hdr, '#include "../potrf_rcwd.cuh"', "namespace bsp {"]
+        for ct in RCW_CT:
+            body.append(f"template cudaError_t launch_rcwd<{n}, {ct}>(const FactorArgs &);")
+            entries.append(f"{{13, {n}, 0, {ct}, 0, &launch_rcwd<{n}, {ct}>}}")
+        body.append("}  // namespace bsp\n")
+        name = f"inst_rcwd_{n:02d}.cu"
         write_if_changed(os.path.join(GEN, name), "\n".join(body))
         files.add(name)
     for n in REGV_N:
