@@ -116,11 +116,18 @@ enum {
                                  the input comes by per-thread copies (chunk
                                  != 32), slower with chunk 32 (TMA path);
                                  any chunk; 49 <= n <= 64                     */
-    BSPOTRF_VARIANT_RCWD = 13  /* RCW plus a ninth warp that factors each 8x8
+    BSPOTRF_VARIANT_RCWD = 13, /* RCW plus a ninth warp that factors each 8x8
                                  diagonal block while the row warps run the
                                  GEMM of their other rows (two passes over the
                                  row buffer); one CTA per SM; any chunk;
                                  49 <= n <= 64                                */
+    BSPOTRF_VARIANT_RCWP = 14  /* "paged" RCW: the factor in 8-column TMEM
+                                 pages recycled as row slots die (at most 128
+                                 columns per warp), one row buffer + stage set
+                                 in shared memory, TWO CTAs per SM (256 TMEM
+                                 columns each); `param` 1 = the 8x8 diagonal
+                                 block factored by one warp (0: by all eight,
+                                 as RCW); any chunk; 33 <= n <= 64            */
 };
 
 /* Launch tuning (a row of the autotuning table). */

@@ -21,7 +21,7 @@ __all__ = [
     "batch_spotrf_interleaved_host", "batch_spotrf_host_bytes",
     "bspotrf_synth_generate", "bspotrf_fill_u32", "bspotrf_probe_copy_lower", "Tuning",
     "batch_interleaved_rhs_elems", "batch_spotrs_interleaved", "batch_sposv_interleaved",
-    "bspotrf_tuning_available", "VARIANT_AUTO", "VARIANT_REG", "VARIANT_SMEM", "VARIANT_TILE", "VARIANT_PANEL", "VARIANT_PTMEM", "VARIANT_RTMA", "VARIANT_RTMAP", "VARIANT_QTM", "VARIANT_REGX", "VARIANT_RCW", "VARIANT_REGV", "VARIANT_RCW16", "VARIANT_RCWD",
+    "bspotrf_tuning_available", "VARIANT_AUTO", "VARIANT_REG", "VARIANT_SMEM", "VARIANT_TILE", "VARIANT_PANEL", "VARIANT_PTMEM", "VARIANT_RTMA", "VARIANT_RTMAP", "VARIANT_QTM", "VARIANT_REGX", "VARIANT_RCW", "VARIANT_REGV", "VARIANT_RCW16", "VARIANT_RCWD", "VARIANT_RCWP",
     "SYNTH_KINDS", "UPPER_MODES", "LIB_PATH",
 ]
 
@@ -29,7 +29,7 @@ LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libbspotrf.
 
 (VARIANT_AUTO, VARIANT_REG, VARIANT_SMEM, VARIANT_TILE, VARIANT_PANEL, VARIANT_PTMEM,
  VARIANT_RTMA, VARIANT_RTMAP, VARIANT_QTM, VARIANT_REGX, VARIANT_RCW, VARIANT_REGV, VARIANT_RCW16,
- VARIANT_RCWD) = 0, 1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11, 12, 13
+ VARIANT_RCWD, VARIANT_RCWP) = 0, 1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11, 12, 13, 14
 SYNTH_KINDS = {"dd": 0, "als": 1, "l0": 2}
 UPPER_MODES = {"mirror": 0, "nan": 1, "keep": 2}
 

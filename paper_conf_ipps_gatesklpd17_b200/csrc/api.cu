@@ -143,6 +143,11 @@ static LaunchFn resolve(int n, int chunk, const bspotrf_tuning &t, int *tpb_out)
         LaunchFn f = find(BSPOTRF_VARIANT_RCWD, n, 0, chunk == 32 ? 32 : 0, 0);
         return f ? f : find(BSPOTRF_VARIANT_RCWD, n, 0, 0, 0);
     }
+    case BSPOTRF_VARIANT_RCWP: {
+        *tpb_out = 256;
+        LaunchFn f = find(BSPOTRF_VARIANT_RCWP, n, t.param, chunk == 32 ? 32 : 0, 0);
+        return f ? f : find(BSPOTRF_VARIANT_RCWP, n, t.param, 0, 0);
+    }
     case BSPOTRF_VARIANT_REGV:
         return find(BSPOTRF_VARIANT_REGV, n, 0, 0, 0);
     case BSPOTRF_VARIANT_RCW: {

@@ -123,6 +123,9 @@ def candidates(n, chunk):
         c.append(dict(variant=bsp.VARIANT_RCW16, threads_per_block=512, param=0, staging=0))
     if n in gen_instances.RCWD_N:
         c.append(dict(variant=bsp.VARIANT_RCWD, threads_per_block=288, param=0, staging=0))
+    if n in gen_instances.RCWP_N:
+        for d1 in (0, 1):
+            c.append(dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0))
     for nb in (2, 4, 8):
         if nb <= n or nb == 2:
             for tpb in (64, 128, 256):
@@ -140,7 +143,7 @@ def main():
     ap.add_argument("--kind", default="dd")
     ap.add_argument("--skip-from", action="append", default=[],
                     help="JSONL files whose points are already measured")
-    ap.add_argument("--variants", default="1,2,3,4,5,6,7,8,10,11,12,13")   # 9 (REGX) on request
+    ap.add_argument("--variants", default="1,2,3,4,5,6,7,8,10,11,12,13,14")   # 9 (REGX) on request
     ap.add_argument("--carveouts", default="0", help="e.g. 0,1,25,50,100")
     ap.add_argument("--only", default=None,
                     help="JSON list of tunings to measure instead of candidates() (e.g. table rows)")

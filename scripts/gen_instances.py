@@ -53,6 +53,7 @@ REGV_N = range(1, 9)
 RCW_N = range(33, 65)
 RCW16_N = range(49, 65)
 RCWD_N = range(49, 65)
+RCWP_N = range(33, 65)
 RCW_CT = (32, 0)
 
 
@@ -329,6 +330,17 @@ def main():
             entries.append(f"{{13, {n}, 0, {ct}, 0, &launch_rcwd<{n}, {ct}>}}")
         body.append("}  // namespace bsp\n")
         name = f"inst_rcwd_{n:02d}.cu"
+        write_if_changed(os.path.join(GEN, name), "\n".join(body))
+        files.add(name)
+    for n in RCWP_N:
+        body = [hdr, '#include "../potrf_rcwp.cuh"', "namespace bsp {"]
+        for d1 in (0, 1):
+            for ct in RCW_CT:
+                b = "true" if d1 else "false"
+                body.append(f"template cudaError_t launch_rcwp<{n}, {ct}, {b}>(const FactorArgs &);")
+                entries.append(f"{{14, {n}, {d1}, {ct}, 0, &launch_rcwp<{n}, {ct}, {b}>}}")
+        body.append("}  // namespace bsp\n")
+        name = f"inst_rcwp_{n:02d}.cu"
         write_if_changed(os.path.join(GEN, name), "\n".join(body))
         files.add(name)
     for n in REGV_N:

@@ -88,7 +88,8 @@ def test_tuning_table_covers_every_n(L):
             assert t.variant in (bsp.VARIANT_REG, bsp.VARIANT_SMEM, bsp.VARIANT_TILE,
                                  bsp.VARIANT_PANEL, bsp.VARIANT_PTMEM, bsp.VARIANT_RTMA,
                                  bsp.VARIANT_RTMAP, bsp.VARIANT_QTM, bsp.VARIANT_REGX,
-                                 bsp.VARIANT_RCW, bsp.VARIANT_REGV, bsp.VARIANT_RCW16, bsp.VARIANT_RCWD)
+                                 bsp.VARIANT_RCW, bsp.VARIANT_REGV, bsp.VARIANT_RCW16, bsp.VARIANT_RCWD,
+                                 bsp.VARIANT_RCWP)
             assert t.threads_per_block % 32 == 0
     with pytest.raises(bsp.BspotrfError):
         bsp.bspotrf_get_tuning(65, 32)

@@ -128,6 +128,8 @@ def test_rcw_parity_failures_ragged(n, chunk):
         ts.append(dict(variant=bsp.VARIANT_RCW16, threads_per_block=512, param=0, staging=0))
     if n in gen_instances_mod().RCWD_N:
         ts.append(dict(variant=bsp.VARIANT_RCWD, threads_per_block=288, param=0, staging=0))
+    if n in gen_instances_mod().RCWP_N:
+        ts += [dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0) for d1 in (0, 1)]
     for t in ts:
         out, info, cnt = run_gpu(n, batch, chunk, inter, tune=t)
         assert np.array_equal(info, np.where(failed, kk + 1, 0)), t
@@ -218,6 +220,8 @@ def _tunings(n, chunk):
         out.append(dict(variant=bsp.VARIANT_RCW16, threads_per_block=512, param=0, staging=0))
     if n in gen_instances_mod().RCWD_N:
         out.append(dict(variant=bsp.VARIANT_RCWD, threads_per_block=288, param=0, staging=0))
+    if n in gen_instances_mod().RCWP_N:
+        out += [dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0) for d1 in (0, 1)]
     if n <= 8:
         out.append(dict(variant=bsp.VARIANT_REGV, threads_per_block=128, param=0, staging=0))
     for tpb in (64, 256):
@@ -309,6 +313,8 @@ def test_rcw_many_groups_per_cta(n, chunk):
         ts.append(dict(variant=bsp.VARIANT_RCW16, threads_per_block=512, param=0, staging=0))
     if n in gen_instances_mod().RCWD_N:
         ts.append(dict(variant=bsp.VARIANT_RCWD, threads_per_block=288, param=0, staging=0))
+    if n in gen_instances_mod().RCWP_N:
+        ts += [dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0) for d1 in (0, 1)]
     idx = np.unique(np.concatenate([np.arange(0, batch, 37), np.arange(batch - 200, batch),
                                     np.arange(0, 64 * 32, 31)]))
     ref = None
