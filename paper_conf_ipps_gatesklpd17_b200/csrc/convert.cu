@@ -24,8 +24,13 @@
 //                        32-bit, one element per lane.
 // The previous version (block-wide smem tile, 32-bit accesses, __syncthreads
 // between load and store phases) reached 2.4-2.9 TB/s (profiles/r01/c4_nsweep_r17.md).
+// Which kernel runs (launch_convert): v1 (below) for the ragged last group and
+// C % 4 != 0; v2 (128-bit both sides, paths A / B / D) for the full groups;
+// v3 (sector-aligned row streams) for interleaved -> canonical at E % 8 != 0,
+// n >= 13 (profiles/r02/convert_v3.md).
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 namespace bsp {
 
@@ -683,6 +688,153 @@ convert2d_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
     }
 }
 
+// ---- v3: interleaved -> canonical, fixed 32-element slices, sector-aligned
+// row streams (round 2) ---------------------------------------------------------
+// Why.  The canonical side of a slice is 32 row segments that start wherever
+// R*E + e0 falls.  When that is not a multiple of 8 floats (odd n, and every
+// odd row at n = 2 mod 4), each segment begins and ends inside a 32-B DRAM
+// sector that another tile (v2 path B: another warp) or a later instruction
+// (convert2d) completes: 0.48-0.64 of HBM against 0.82-0.85 for n = 0 mod 4
+// (j13 A/B).  Here a group row is cut into FIXED 32-element slices e0 = 32k
+// (the last one E - 32(K-1) wide) and every row's tile is shifted by its
+// SECTOR phase ph = (R*E) mod 8: tile x = ph + li, so tile x = 0 is a sector
+// start of the canonical stream.  A slice then writes, per row, 4 whole sectors
+// (x = 0..31) -- each sector as two adjacent lanes' float4s in ONE instruction
+// -- and keeps x = 32..32+ph-1 (< 8 floats) as the carry that becomes x < ph
+// of the next slice.  Only a unit's first partial sector and its last partial
+// one are stored as scalars.  Phases are per-lane constants (fixed slices):
+//   line side  (lane = l8 + 8*lq): rows 4*l8 + j, element li = 4*kk + lq;
+//   slot side  rows lq + 4*k, float4 slot l8 (x = 4*l8..+3): ph takes two
+//              values, by the parity of k (4*k*E mod 8);
+//   carry      slots 8, 9 of row = lane.
+// Physical slot = logical ^ (row >> 2) for slots 0..7 (a quarter warp reads a
+// row's 8 slots: conflict-free), slots 8, 9 unswizzled.  A work unit is slices
+// [k0, k1) of one 32-matrix group (S segments per group: >= 16 units per warp);
+// persistent warps, the next slice's loads in flight during the stores.
+constexpr int CV3_P = 40;                                  // 10 float4 slots per tile row
+constexpr int CV3_WARP = 32 * CV3_P;
+
+struct Cv3Shape {
+    int64_t C, G, units;
+    int E, K, WL, S;       // slices per row, last slice width, segments per group
+};
+
+__device__ __forceinline__ int cv3_swz(int a, int f) { return a < 8 ? (a ^ f) : a; }
+
+__global__ void __launch_bounds__(CV_THREADS, 3)
+convert3_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv3Shape s) {
+    extern __shared__ __align__(16) float cv3_smem[];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    float *T = cv3_smem + wid * CV3_WARP;
+    const int64_t W = (int64_t)gridDim.x * CV_WARPS;
+    int64_t u = (int64_t)blockIdx.x * CV_WARPS + wid;
+    if (u >= s.units) return;
+    const int E = s.E;
+    const int l8 = lane & 7, lq = lane >> 3, c4 = 4 * l8;
+    int lb[4], hb[4];                                      // line side, rows c4 + j
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        const int x0 = (((c4 + j) * E) & 7) + lq;
+        lb[j] = (c4 + j) * CV3_P + (x0 & 3);
+        hb[j] = x0 >> 2;
+    }
+    // slot side, rows lq + 4k: phase by the parity of k
+    const int ph0 = (lq * E) & 7, ph1 = (lq * E + 4 * E) & 7;
+    float *Ts = T + lq * CV3_P;
+    const int64_t so0 = (int64_t)lq * E - ph0 + 4 * l8, so1 = (int64_t)lq * E - ph1 + 4 * l8;
+    const int phc = (lane * E) & 7;                        // carry lane: row = lane
+    float *T8 = T + lane * CV3_P + 32;
+    float *T0 = T + lane * CV3_P + 4 * (lane >> 2);        // logical slots 0, 1 of the row
+    float *T1 = T + lane * CV3_P + 4 * (1 ^ (lane >> 2));
+    const int64_t coff = (int64_t)lane * E - phc + 32;
+
+    auto unit = [&](int64_t uu, int64_t &g, int &k0, int &k1) {
+        g = uu / s.S;
+        const int sg = (int)(uu - g * s.S);
+        k0 = (int)((int64_t)sg * s.K / s.S);
+        k1 = (int)((int64_t)(sg + 1) * s.K / s.S);
+    };
+    auto width = [&](int k) { return k == s.K - 1 ? s.WL : 32; };
+    auto lines = [&](int64_t g) {                          // interleaved offset of the group's lane 0
+        const int64_t m0 = g * 32;
+        return (m0 / s.C) * s.C * (int64_t)E + m0 % s.C;
+    };
+    float4 R4[8];
+    auto load = [&](int64_t g, int k) {                    // interleaved lines e0 + 4kk + lq
+        const int w = width(k);
+        const float *lp = src + lines(g) + (int64_t)(32 * k + lq) * s.C + c4;
+#pragma unroll
+        for (int kk = 0; kk < 8; ++kk)
+            if (4 * kk + lq < w) R4[kk] = ldg4(lp + (int64_t)(4 * kk) * s.C);
+    };
+
+    int64_t g;
+    int k0, k1;
+    unit(u, g, k0, k1);
+    int k = k0;
+    load(g, k);
+    for (;;) {
+        const int w = width(k), e0 = 32 * k;
+        const bool first = k == k0, last = k == k1 - 1;
+#pragma unroll
+        for (int kk = 0; kk < 8; ++kk)                     // lines -> tile rows (x = ph + li)
+            if (4 * kk + lq < w) {
+                const float v[4] = {R4[kk].x, R4[kk].y, R4[kk].z, R4[kk].w};
+#pragma unroll
+                for (int j = 0; j < 4; ++j) T[lb[j] + 4 * cv3_swz(hb[j] + kk, l8)] = v[j];
+            }
+        __syncwarp();
+        // next slice (or the next unit's first) in flight during the stores
+        int64_t gn = g;
+        int kn = k + 1, k0n = k0, k1n = k1;
+        bool more = true;
+        if (last) {
+            u += W;
+            more = u < s.units;
+            if (more) unit(u, gn, k0n, k1n);
+            kn = k0n;
+        }
+        if (more) load(gn, kn);
+        // tile -> canonical: slots 0..7 of rows lq + 4k8 (x valid in [lo, hi))
+        float *cp = dst + g * 32 * (int64_t)E + e0;
+#pragma unroll
+        for (int k8 = 0; k8 < 8; ++k8) {
+            const int ph = (k8 & 1) ? ph1 : ph0;
+            const int x0 = 4 * l8;
+            const int lo = first ? min(max(ph - x0, 0), 4) : 0;
+            const int hi = last ? min(max(ph + w - x0, 0), 4) : 4;
+            const float4 q = *reinterpret_cast<const float4 *>(Ts + k8 * 4 * CV3_P + 4 * (l8 ^ k8));
+            float *p = cp + ((k8 & 1) ? so1 : so0) + (int64_t)(4 * k8) * E;
+            if (lo == 0 && hi == 4) {
+                stg4(p, q.x, q.y, q.z, q.w);
+            } else {
+                const float v[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+                for (int jj = 0; jj < 4; ++jj)
+                    if (jj >= lo && jj < hi) stg1(p + jj, v[jj]);
+            }
+        }
+        __syncwarp();                                      // slots 0, 1 read before the carry lands
+        if (!last) {                                       // carry: x = 32..32+phc-1 -> x < phc
+            if (phc) {
+                *reinterpret_cast<float4 *>(T0) = *reinterpret_cast<const float4 *>(T8);
+                if (phc > 4) *reinterpret_cast<float4 *>(T1) = *reinterpret_cast<const float4 *>(T8 + 4);
+            }
+        } else if (32 < phc + w) {                         // the unit ends inside x = 32..39
+            const int rm = phc + w - 32;
+#pragma unroll
+            for (int jj = 0; jj < 7; ++jj)
+                if (jj < rm) stg1(cp + coff + jj, T8[jj]);
+        }
+        if (!more) break;
+        __syncwarp();
+        g = gn;
+        k = kn;
+        k0 = k0n;
+        k1 = k1n;
+    }
+}
+
 template <typename K>
 static cudaError_t launch_persistent(K kern, int64_t tiles, const float *src, float *dst, const Cv2Shape &s,
                                      cudaStream_t stream, size_t dyn_smem = 0) {
@@ -752,6 +904,43 @@ static cudaError_t launch_v2(int n, int64_t G, int64_t C, const float *src, floa
     return cudaErrorInvalidValue;
 }
 
+static cudaError_t launch_v3(int n, int64_t G, int64_t C, const float *src, float *dst, cudaStream_t stream) {
+    Cv3Shape s;
+    s.C = C;
+    s.G = G;
+    s.E = n * n;
+    s.K = (s.E + 31) / 32;
+    s.WL = s.E - 32 * (s.K - 1);
+    auto kern = convert3_kernel;
+    constexpr size_t SMEM = (size_t)CV_WARPS * CV3_WARP * sizeof(float);
+    int dev = 0, sms = 148, per_sm = 3;
+    if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
+    if (e != cudaSuccess) return e;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, CV_THREADS, SMEM);
+    if (per_sm < 1) per_sm = 1;
+    int64_t grid = (int64_t)sms * per_sm;
+    // segments per group: >= 16 units per warp (balance), at most one per slice
+    const int64_t warps = grid * CV_WARPS;
+    int64_t S = (16 * warps + G - 1) / G;
+    if (S > s.K) S = s.K;
+    if (S < 1) S = 1;
+    s.S = (int)S;
+    s.units = G * S;
+    const int64_t need = (s.units + CV_WARPS - 1) / CV_WARPS;
+    if (grid > need) grid = need;
+    kern<<<(unsigned)grid, CV_THREADS, SMEM, stream>>>(src, dst, s);
+    return cudaGetLastError();
+}
+
+// v3 (fixed slices, constant phases) vs v2, per direction and n: see the
+// choice in launch_convert.  BSPOTRF_CONVERT_PATH=v2|v3 forces one (probes).
+static int convert_path_override() {
+    const char *v = getenv("BSPOTRF_CONVERT_PATH");
+    if (!v) return 0;
+    return (v[0] == 'v' && v[1] == '3') ? 3 : ((v[0] == 'v' && v[1] == '2') ? 2 : 0);
+}
+
 cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float *src, float *dst,
                            cudaStream_t stream) {
     // n = 1: element (0,0) of matrix b sits at offset b in BOTH layouts
@@ -765,8 +954,16 @@ cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float
     if (v2) {
         const int64_t G = batch / 32;
         if (G > 0) {
-            const cudaError_t e = dir == 0 ? launch_v2<0>(n, G, C, src, dst, stream)
-                                           : launch_v2<1>(n, G, C, src, dst, stream);
+            const int ov = convert_path_override();
+            const int E = n * n;
+            // interleaved -> canonical: v3 where v2's canonical rows are not
+            // 32-B aligned (E % 8 != 0) and rows span >= 6 slices (n >= 13; at
+            // n = 6..11 the partial first / last sectors of the few slices per
+            // row cost more than they save: j13b A/B, profiles/r02/convert_v3.md)
+            const bool v3 = dir == 1 && E > 32 && (ov == 3 || (ov == 0 && E % 8 != 0 && n >= 13));
+            const cudaError_t e = v3 ? launch_v3(n, G, C, src, dst, stream)
+                                     : (dir == 0 ? launch_v2<0>(n, G, C, src, dst, stream)
+                                                 : launch_v2<1>(n, G, C, src, dst, stream));
             if (e != cudaSuccess) return e;
         }
         gbeg = G;

@@ -12,7 +12,7 @@ from gpu_helpers import assert_parity, make_batch, run_gpu, torch_mod
 pytestmark = pytest.mark.gpu
 
 
-@pytest.mark.parametrize("n", [1, 2, 3, 4, 5, 6, 7, 8, 9, 12, 16, 31, 32, 33, 45, 63, 64])
+@pytest.mark.parametrize("n", [1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 12, 14, 16, 31, 32, 33, 45, 50, 63, 64])
 @pytest.mark.parametrize("chunk", [32, 64, 0, 160])
 @pytest.mark.parametrize("batch", [517, 1024, 96, 1, 1184, 1002])
 def test_conversion_matches_layout_definition(n, chunk, batch):
@@ -36,6 +36,42 @@ def test_conversion_matches_layout_definition(n, chunk, batch):
     back = torch.full((batch * n * n,), 7.0, device="cuda")
     bsp.batch_interleaved_to_canonical(n, batch, chunk, ddst, back)
     assert np.array_equal(back.cpu().numpy().view(np.uint32), canon.reshape(-1).view(np.uint32))
+
+
+def _roundtrip_exact(n, batch, chunk, seed):
+    torch = torch_mod()
+    rng = np.random.default_rng(seed)
+    canon = rng.standard_normal((batch, n * n), dtype=np.float32)
+    expect = layout.to_interleaved(n, chunk, canon, fill_bits=synth.PAD_BITS)
+    dsrc = torch.from_numpy(canon).cuda()
+    ddst = torch.zeros(expect.size, dtype=torch.float32, device="cuda")
+    bsp.bspotrf_fill_u32(ddst, synth.PAD_BITS)
+    bsp.batch_canonical_to_interleaved(n, batch, chunk, dsrc, ddst)
+    assert np.array_equal(ddst.cpu().numpy().view(np.uint32), expect.view(np.uint32))
+    back = torch.full((batch * n * n,), 7.0, device="cuda")
+    bsp.batch_interleaved_to_canonical(n, batch, chunk, ddst, back)
+    assert np.array_equal(back.cpu().numpy().view(np.uint32), canon.reshape(-1).view(np.uint32))
+
+
+@pytest.mark.parametrize("path", ["v3", "v2"])
+@pytest.mark.parametrize("n", [6, 7, 10, 11, 12, 14, 17, 18, 30, 33, 34, 50, 61, 62, 64])
+@pytest.mark.parametrize("chunk,batch", [(32, 1184), (0, 9632), (96, 4096 + 32 * 7 + 5)])
+def test_conversion_paths_forced(monkeypatch, path, n, chunk, batch):
+    """v3 (fixed 32-element slices, per-lane constant row phases, carries between
+    slices) and v2 (proportional / aligned slices), each forced on every n
+    class -- E % 4 in {0, 1}, E % 8 in {0, 4}, the last slice 1..32 wide -- with
+    small group counts, where every group is cut into many segments (a unit =
+    a few slices: partial first / last slots stored by scalars)."""
+    monkeypatch.setenv("BSPOTRF_CONVERT_PATH", path)
+    _roundtrip_exact(n, batch, chunk, seed=n * 7 + chunk)
+
+
+@pytest.mark.parametrize("n,batch", [(7, 1 << 21), (10, 1 << 20), (63, 1 << 16), (62, 3 * 1 << 15)])
+def test_conversion_large_batch(n, batch):
+    """Default paths at batches where v3 runs one or two segments per group
+    (whole-row streams with carries across every slice) and every persistent
+    warp loops over many units."""
+    _roundtrip_exact(n, batch, 32, seed=n)
 
 
 @pytest.mark.parametrize("kind", ["dd", "als", "l0"])
