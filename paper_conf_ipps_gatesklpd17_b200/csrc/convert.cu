@@ -707,128 +707,146 @@ convert2d_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
 //   slot side  rows lq + 4*k, float4 slot l8 (x = 4*l8..+3): ph takes two
 //              values, by the parity of k (4*k*E mod 8);
 //   carry      slots 8, 9 of row = lane.
-// Physical slot = logical ^ (row >> 2) for slots 0..7 (a quarter warp reads a
-// row's 8 slots: conflict-free), slots 8, 9 unswizzled.  A work unit is slices
-// [k0, k1) of one 32-matrix group (S segments per group: >= 16 units per warp);
-// persistent warps, the next slice's loads in flight during the stores.
-constexpr int CV3_P = 40;                                  // 10 float4 slots per tile row
-constexpr int CV3_WARP = 32 * CV3_P;
+// Shared tile: row R starts at R*P + 4*t(R >> 2) (rows 16-B aligned, x =
+// 0..39 used); the per-row shift t and pitch P depend only on the class of E
+// mod 8 (odd n: 1, n = 2 mod 4: 4) and make the line side conflict-free (the 8
+// rows 4*l8 + j of one STS hit 8 disjoint 4-bank groups; found by exhaustive
+// search); the slot side reads one row's 8 contiguous slots per quarter warp.
+// All tile addresses are a per-lane base + a compile-time immediate.  (A first
+// version with XOR-swizzled slots ran 765 warp instructions per 4-KB slice,
+// IMAD/LOP3/LEA 58% of them, and 2.4-way conflicts on the line side: j14 ncu.)
+// A work unit is slices [k0, k1) of one 32-matrix group (S segments per group:
+// >= 16 units per warp); persistent warps, the next slice's loads in flight
+// during the stores.
+template <int EC>
+struct Cv3Tile {
+    static constexpr int P = EC == 1 ? 60 : 52;
+    // t(l8), 4 bits each: E = 1 mod 8: 0,0,1,1,3,2,4,5; E = 4 mod 8: 0,0,1,1,2,2,3,3
+    static constexpr uint32_t TP = EC == 1 ? 0x54231100u : 0x33221100u;
+    __host__ __device__ static constexpr int t(int q) { return (int)((TP >> (4 * q)) & 15u); }
+    __host__ __device__ static constexpr int row(int R) { return R * P + 4 * t(R >> 2); }
+    static constexpr int WARP = 32 * P;
+};
 
 struct Cv3Shape {
     int64_t C, G, units;
     int E, K, WL, S;       // slices per row, last slice width, segments per group
 };
 
-__device__ __forceinline__ int cv3_swz(int a, int f) { return a < 8 ? (a ^ f) : a; }
-
+template <int EC>
 __global__ void __launch_bounds__(CV_THREADS, 3)
 convert3_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv3Shape s) {
+    using TT = Cv3Tile<EC>;
     extern __shared__ __align__(16) float cv3_smem[];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    float *T = cv3_smem + wid * CV3_WARP;
+    float *T = cv3_smem + wid * TT::WARP;
     const int64_t W = (int64_t)gridDim.x * CV_WARPS;
     int64_t u = (int64_t)blockIdx.x * CV_WARPS + wid;
     if (u >= s.units) return;
     const int E = s.E;
     const int l8 = lane & 7, lq = lane >> 3, c4 = 4 * l8;
-    int lb[4], hb[4];                                      // line side, rows c4 + j
+    // line side: rows 4*l8 + j, element 4*kk + lq at tile x = ph + 4*kk + lq
+    float *Tl[4];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-        const int x0 = (((c4 + j) * E) & 7) + lq;
-        lb[j] = (c4 + j) * CV3_P + (x0 & 3);
-        hb[j] = x0 >> 2;
-    }
-    // slot side, rows lq + 4k: phase by the parity of k
+    for (int j = 0; j < 4; ++j) Tl[j] = T + TT::row(c4 + j) + (((c4 + j) * E) & 7) + lq;
+    // slot side: rows lq + 4*k8 (row offset lq*P + compile-time), slot l8; the
+    // sector phase of the row takes two values, by the parity of k8
+    float *Ts = T + lq * TT::P + 4 * l8;
     const int ph0 = (lq * E) & 7, ph1 = (lq * E + 4 * E) & 7;
-    float *Ts = T + lq * CV3_P;
-    const int64_t so0 = (int64_t)lq * E - ph0 + 4 * l8, so1 = (int64_t)lq * E - ph1 + 4 * l8;
-    const int phc = (lane * E) & 7;                        // carry lane: row = lane
-    float *T8 = T + lane * CV3_P + 32;
-    float *T0 = T + lane * CV3_P + 4 * (lane >> 2);        // logical slots 0, 1 of the row
-    float *T1 = T + lane * CV3_P + 4 * (1 ^ (lane >> 2));
-    const int64_t coff = (int64_t)lane * E - phc + 32;
+    const int so0 = lq * E - ph0 + 4 * l8, so1 = lq * E - ph1 + 4 * l8;
+    // carry lane: row = lane, x = 32..39 -> x = 0..7
+    const int phc = (lane * E) & 7;
+    float *T8 = T + lane * TT::P + 4 * (int)((TT::TP >> (4 * (lane >> 2))) & 15u);
+    const int coff = lane * E - phc + 32;
+    const int64_t C4 = 4 * s.C;
 
-    auto unit = [&](int64_t uu, int64_t &g, int &k0, int &k1) {
+    // a unit: group g, slices [k0, k1), interleaved offset lb of the group's lane 0
+    auto unit = [&](int64_t uu, int64_t &g, int &k0, int &k1, int64_t &lb) {
         g = uu / s.S;
         const int sg = (int)(uu - g * s.S);
         k0 = (int)((int64_t)sg * s.K / s.S);
         k1 = (int)((int64_t)(sg + 1) * s.K / s.S);
-    };
-    auto width = [&](int k) { return k == s.K - 1 ? s.WL : 32; };
-    auto lines = [&](int64_t g) {                          // interleaved offset of the group's lane 0
         const int64_t m0 = g * 32;
-        return (m0 / s.C) * s.C * (int64_t)E + m0 % s.C;
+        lb = (m0 / s.C) * s.C * (int64_t)E + m0 % s.C;
     };
     float4 R4[8];
-    auto load = [&](int64_t g, int k) {                    // interleaved lines e0 + 4kk + lq
-        const int w = width(k);
-        const float *lp = src + lines(g) + (int64_t)(32 * k + lq) * s.C + c4;
+    auto load = [&](int64_t lb, int k) {                   // interleaved lines 32k + 4kk + lq
+        const int w = k == s.K - 1 ? s.WL : 32;
+        const float *lp = src + lb + (int64_t)(32 * k + lq) * s.C + c4;
 #pragma unroll
-        for (int kk = 0; kk < 8; ++kk)
-            if (4 * kk + lq < w) R4[kk] = ldg4(lp + (int64_t)(4 * kk) * s.C);
+        for (int kk = 0; kk < 8; ++kk) {
+            if (4 * kk + lq < w) R4[kk] = ldg4(lp);
+            lp += C4;
+        }
     };
 
-    int64_t g;
+    int64_t g, lb;
     int k0, k1;
-    unit(u, g, k0, k1);
+    unit(u, g, k0, k1, lb);
     int k = k0;
-    load(g, k);
+    load(lb, k);
     for (;;) {
-        const int w = width(k), e0 = 32 * k;
+        const int w = k == s.K - 1 ? s.WL : 32, e0 = 32 * k;
         const bool first = k == k0, last = k == k1 - 1;
 #pragma unroll
-        for (int kk = 0; kk < 8; ++kk)                     // lines -> tile rows (x = ph + li)
+        for (int kk = 0; kk < 8; ++kk)                     // lines -> tile rows
             if (4 * kk + lq < w) {
-                const float v[4] = {R4[kk].x, R4[kk].y, R4[kk].z, R4[kk].w};
-#pragma unroll
-                for (int j = 0; j < 4; ++j) T[lb[j] + 4 * cv3_swz(hb[j] + kk, l8)] = v[j];
+                Tl[0][4 * kk] = R4[kk].x;
+                Tl[1][4 * kk] = R4[kk].y;
+                Tl[2][4 * kk] = R4[kk].z;
+                Tl[3][4 * kk] = R4[kk].w;
             }
         __syncwarp();
         // next slice (or the next unit's first) in flight during the stores
-        int64_t gn = g;
+        int64_t gn = g, lbn = lb;
         int kn = k + 1, k0n = k0, k1n = k1;
         bool more = true;
         if (last) {
             u += W;
             more = u < s.units;
-            if (more) unit(u, gn, k0n, k1n);
+            if (more) unit(u, gn, k0n, k1n, lbn);
             kn = k0n;
         }
-        if (more) load(gn, kn);
-        // tile -> canonical: slots 0..7 of rows lq + 4k8 (x valid in [lo, hi))
+        if (more) load(lbn, kn);
+        // tile -> canonical: slot l8 of rows lq + 4k8, x valid in [lo, hi)
         float *cp = dst + g * 32 * (int64_t)E + e0;
+        int lo[2], hi[2];
+#pragma unroll
+        for (int pp = 0; pp < 2; ++pp) {
+            const int ph = pp ? ph1 : ph0;
+            lo[pp] = first ? min(max(ph - c4, 0), 4) : 0;
+            hi[pp] = last ? min(max(ph + w - c4, 0), 4) : 4;
+        }
 #pragma unroll
         for (int k8 = 0; k8 < 8; ++k8) {
-            const int ph = (k8 & 1) ? ph1 : ph0;
-            const int x0 = 4 * l8;
-            const int lo = first ? min(max(ph - x0, 0), 4) : 0;
-            const int hi = last ? min(max(ph + w - x0, 0), 4) : 4;
-            const float4 q = *reinterpret_cast<const float4 *>(Ts + k8 * 4 * CV3_P + 4 * (l8 ^ k8));
-            float *p = cp + ((k8 & 1) ? so1 : so0) + (int64_t)(4 * k8) * E;
-            if (lo == 0 && hi == 4) {
+            const float4 q = *reinterpret_cast<const float4 *>(Ts + 4 * k8 * TT::P + 4 * TT::t(k8));
+            float *p = cp + ((k8 & 1) ? so1 : so0) + 4 * k8 * E;
+            const int a = lo[k8 & 1], b = hi[k8 & 1];
+            if (a == 0 && b == 4) {
                 stg4(p, q.x, q.y, q.z, q.w);
             } else {
                 const float v[4] = {q.x, q.y, q.z, q.w};
 #pragma unroll
                 for (int jj = 0; jj < 4; ++jj)
-                    if (jj >= lo && jj < hi) stg1(p + jj, v[jj]);
+                    if (jj >= a && jj < b) stg1(p + jj, v[jj]);
             }
         }
         __syncwarp();                                      // slots 0, 1 read before the carry lands
         if (!last) {                                       // carry: x = 32..32+phc-1 -> x < phc
             if (phc) {
-                *reinterpret_cast<float4 *>(T0) = *reinterpret_cast<const float4 *>(T8);
-                if (phc > 4) *reinterpret_cast<float4 *>(T1) = *reinterpret_cast<const float4 *>(T8 + 4);
+                *reinterpret_cast<float4 *>(T8) = *reinterpret_cast<const float4 *>(T8 + 32);
+                if (phc > 4) *reinterpret_cast<float4 *>(T8 + 4) = *reinterpret_cast<const float4 *>(T8 + 36);
             }
         } else if (32 < phc + w) {                         // the unit ends inside x = 32..39
             const int rm = phc + w - 32;
 #pragma unroll
             for (int jj = 0; jj < 7; ++jj)
-                if (jj < rm) stg1(cp + coff + jj, T8[jj]);
+                if (jj < rm) stg1(cp + coff + jj, T8[32 + jj]);
         }
         if (!more) break;
         __syncwarp();
         g = gn;
+        lb = lbn;
         k = kn;
         k0 = k0n;
         k1 = k1n;
@@ -904,6 +922,7 @@ static cudaError_t launch_v2(int n, int64_t G, int64_t C, const float *src, floa
     return cudaErrorInvalidValue;
 }
 
+template <int EC>
 static cudaError_t launch_v3(int n, int64_t G, int64_t C, const float *src, float *dst, cudaStream_t stream) {
     Cv3Shape s;
     s.C = C;
@@ -911,8 +930,8 @@ static cudaError_t launch_v3(int n, int64_t G, int64_t C, const float *src, floa
     s.E = n * n;
     s.K = (s.E + 31) / 32;
     s.WL = s.E - 32 * (s.K - 1);
-    auto kern = convert3_kernel;
-    constexpr size_t SMEM = (size_t)CV_WARPS * CV3_WARP * sizeof(float);
+    auto kern = convert3_kernel<EC>;
+    constexpr size_t SMEM = (size_t)CV_WARPS * Cv3Tile<EC>::WARP * sizeof(float);
     int dev = 0, sms = 148, per_sm = 3;
     if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM);
@@ -957,11 +976,13 @@ cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float
             const int ov = convert_path_override();
             const int E = n * n;
             // interleaved -> canonical: v3 where v2's canonical rows are not
-            // 32-B aligned (E % 8 != 0) and rows span >= 6 slices (n >= 13; at
-            // n = 6..11 the partial first / last sectors of the few slices per
-            // row cost more than they save: j13b A/B, profiles/r02/convert_v3.md)
-            const bool v3 = dir == 1 && E > 32 && (ov == 3 || (ov == 0 && E % 8 != 0 && n >= 13));
-            const cudaError_t e = v3 ? launch_v3(n, G, C, src, dst, stream)
+            // 32-B aligned (E % 8 != 0) and rows span enough slices (odd n >= 13,
+            // n = 2 mod 4 >= 10; below, the partial first / last sectors of the
+            // few slices per row cost more than they save: profiles/r02/convert_v3.md)
+            const bool v3 = dir == 1 && E > 32 && E % 8 != 0 &&
+                            (ov == 3 || (ov == 0 && n >= (E % 8 == 1 ? 13 : 10)));
+            const cudaError_t e = v3 ? (E % 8 == 1 ? launch_v3<1>(n, G, C, src, dst, stream)
+                                                   : launch_v3<4>(n, G, C, src, dst, stream))
                                      : (dir == 0 ? launch_v2<0>(n, G, C, src, dst, stream)
                                                  : launch_v2<1>(n, G, C, src, dst, stream));
             if (e != cudaSuccess) return e;

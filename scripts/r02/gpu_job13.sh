@@ -19,6 +19,9 @@ ptests)
 tests)
   timeout 2400 python -m pytest tests -m gpu -q -p no:cacheprovider -x > $O/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> $O/pytest_gpu.log
   tail -n 3 $O/pytest_gpu.log ;;
+ncuconv)
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:convert -c 4 -o $O/prof_conv -f \
+    python scripts/r02/conv_probe.py 63 62 > $O/ncu_conv.log 2>&1; echo "ncuconv rc=$?" ;;
 esac; done
 [ -f $O/conv_ab.jsonl ] && python - "$O" <<'PY'
 import json, sys
