@@ -154,7 +154,7 @@ potrf_rcwp_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__
 
     // input of column block c of group g -> units c..R-1: element (i, 8c+w) at
     // [w][i - 8c][q] (RCW's stage layout); lower part only
-    auto prefetch = [&](auto c_, int64_t g) {
+    auto prefetch = [&](auto c_, int64_t g, const float *gb) {
         constexpr int c = BSP_CI(c_);
         float *stg = smf + (size_t)c * UNIT;
         if constexpr (TMA) {
@@ -175,16 +175,26 @@ potrf_rcwp_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__
         } else {
             if (g * 32 + 31 < batch && cs % 4 == 0) {
                 // full group: element (i, j) of the 32 matrices is one 128-B line;
-                // 8 lanes x 16 B per line, 4 lines per warp instruction (RCW's form)
-                const float *gb = A + ((g * 32) / cs) * cs * (int64_t)(N * N) + (g * 32) % cs;
+                // 8 lanes x 16 B per line, 4 lines per warp instruction (RCW's form).
+                // Step tt covers r = c + tt/2, w = sub + 4 (tt & 1): two running
+                // pointers (w = sub, sub + 4) advanced by 8 rows per r -- no 64-bit
+                // products or divisions per copy (the runtime-chunk instances
+                // spilled 36-232 B at 128 registers with the per-copy form)
                 const int l8 = q & 7, sub = q >> 3;
+                const int64_t rstep = 8 * cs;
+                const float *pa = gb + (int64_t)(8 * c + h + (8 * c + sub) * N) * cs + 4 * l8;
+                const float *pb = pa + (int64_t)(4 * N) * cs;
+                float *sa = stg + (sub * RS::rs(c) + h) * 32 + 4 * l8;
+                float *sb = sa + 4 * RS::rs(c) * 32;
 #pragma unroll
-                for (int tt = 0; tt < 2 * (R - c); ++tt) {
-                    const int idx = 4 * tt + sub, r = c + (idx >> 3), w = idx & 7;
-                    const int i = 8 * r + h;
-                    if (i < N && 8 * c + w < N && (r > c || w <= h))
-                        cp_async16(stg + (w * RS::rs(c) + i - 8 * c) * 32 + 4 * l8,
-                                   gb + (int64_t)(i + (8 * c + w) * N) * cs + 4 * l8);
+                for (int rr = 0; rr < R - c; ++rr) {
+                    const int r = c + rr, i = 8 * r + h;
+                    if (i < N) {
+                        if (8 * c + sub < N && (r > c || sub <= h)) cp_async16(sa + 8 * rr * 32, pa);
+                        if (8 * c + sub + 4 < N && (r > c || sub + 4 <= h)) cp_async16(sb + 8 * rr * 32, pb);
+                    }
+                    pa += rstep;
+                    pb += rstep;
                 }
             } else {
                 const int64_t gm = g * 32 + q;
@@ -206,13 +216,16 @@ potrf_rcwp_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__
 
     int64_t g = blockIdx.x;
     uint32_t par = 0;
-    if (g < ngroups) prefetch(std::integral_constant<int, 0>{}, g);
+    // interleaved base of group g's lane 0 (runtime-chunk form)
+    auto gbase = [&](int64_t gg) { return A + ((gg * 32) / cs) * cs * (int64_t)(N * N) + (gg * 32) % cs; };
+    if (g < ngroups) prefetch(std::integral_constant<int, 0>{}, g, TMA ? A : gbase(g));
 
     float acc[R][8];
     for (; g < ngroups; g += gridDim.x) {
         const int64_t gm = g * 32 + q;
         const bool active = gm < batch;
         const Addr<N, CT> ad(A, active ? gm : batch - 1, cs);
+        const float *gb = TMA ? A : gbase(g);
         int inf = 0;
         sfor<0, R>([&](auto c_) {
             constexpr int c = BSP_CI(c_);
@@ -236,7 +249,7 @@ potrf_rcwp_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__
                 });
             }
             __syncthreads();                             // B1
-            if constexpr (c + 1 < R) prefetch(std::integral_constant<int, c + 1>{}, g);
+            if constexpr (c + 1 < R) prefetch(std::integral_constant<int, c + 1>{}, g, gb);
 
             // (b) acc(r) -= L(8r+h, 0..8c-1) L(8c..8c+7, 0..8c-1)^T, k ascending.
             //     a operand: 4 columns of page (r, kq / 2) of TMEM; b operand: RB(c)
@@ -375,7 +388,7 @@ potrf_rcwp_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__
                 rb_put(smf, 2 * c, h, q, &acc[c + 1][0]);
                 rb_put(smf, 2 * c + 1, h, q, &acc[c + 1][4]);
             } else if (g + gridDim.x < ngroups) {
-                prefetch(std::integral_constant<int, 0>{}, g + gridDim.x);
+                prefetch(std::integral_constant<int, 0>{}, g + gridDim.x, TMA ? A : gbase(g + gridDim.x));
             }
         });
         if (active && h == 0) info[gm] = inf;

@@ -88,7 +88,7 @@ def main():
         print("| n | chunk | variant | default | 1% | 25% | 50% | 100% | best / default |")
         print("|---|---|---|---|---|---|---|---|---|")
         V = {1: "REG", 2: "SMEM", 3: "TILE", 4: "PANEL", 5: "PTMEM", 6: "RTMA", 7: "RTMAP", 8: "QTM",
-             9: "REGX", 10: "RCW", 11: "REGV", 12: "RCW16"}
+             9: "REGX", 10: "RCW", 11: "REGV", 12: "RCW16", 13: "RCWD", 14: "RCWP"}
         for k, d in sorted(by.items()):
             if len(d) < 5:
                 continue

@@ -11,11 +11,11 @@ import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 V = {1: "REG", 2: "SMEM", 3: "TILE", 4: "PANEL", 5: "PTMEM", 6: "RTMA", 7: "RTMAP", 8: "QTM",
-     9: "REGX", 10: "RCW", 11: "REGV", 12: "RCW16", 13: "RCWD"}
+     9: "REGX", 10: "RCW", 11: "REGV", 12: "RCW16", 13: "RCWD", 14: "RCWP"}
 KNAME = {1: "potrf_reg_kernel", 2: "potrf_smem_kernel", 3: "potrf_tile_kernel", 4: "potrf_panel_kernel",
          5: "potrf_ptmem_kernel", 6: "potrf_regtma_kernel", 7: "potrf_rtmap_kernel", 8: "potrf_qtm_kernel",
          9: "potrf_regx_kernel", 10: "potrf_rcw_kernel", 11: "potrf_regv_kernel", 12: "potrf_rcw16_kernel",
-         13: "potrf_rcwd_kernel"}
+         13: "potrf_rcwd_kernel", 14: "potrf_rcwp_kernel"}
 
 
 def parse(path):
@@ -80,6 +80,8 @@ def main():
             want = [n, 32 if c == 32 else 0, e["param"]]
         elif v in (12, 13):
             want = [n, 32 if c == 32 else 0]
+        elif v == 14:                             # <N, CT, D1>
+            want = [n, 32 if c == 32 else 0, e["param"]]
         elif v == 9:
             want = [n, e["param"], e["staging"]]
         elif v in (6, 7, 3):

@@ -38,7 +38,7 @@ for n in ns:
 json.dump({"source": f"B200 autotune sweep {src}", "entries": entries}, open(out_table, "w"), indent=1)
 print(f"{len(entries)} rows -> {out_table}")
 if out_md:
-    V = {1: "REG", 2: "SMEM", 3: "TILE", 4: "PANEL", 5: "PTMEM", 6: "RTMA", 7: "RTMAP", 8: "QTM", 9: "REGX", 10: "RCW", 11: "REGV", 12: "RCW16"}
+    V = {1: "REG", 2: "SMEM", 3: "TILE", 4: "PANEL", 5: "PTMEM", 6: "RTMA", 7: "RTMAP", 8: "QTM", 9: "REGX", 10: "RCW", 11: "REGV", 12: "RCW16", 13: "RCWD", 14: "RCWP"}
     with open(out_md, "w") as f:
         f.write("| n | best chunk | variant | tpb | param | staging | ms (1M) | GB/s | Gflop/s | "
                 "best chunk=0 GB/s | 32 | 64 | 128 | 256 | 512 |\n|---|---|---|---|---|---|---|---|---|---|---|---|---|---|---|\n")

@@ -7,7 +7,7 @@ import json
 import sys
 
 V = {1: "REG", 2: "SMEM", 3: "TILE", 4: "PANEL", 5: "PTMEM", 6: "RTMA", 7: "RTMAP", 8: "QTM",
-     9: "REGX", 10: "RCW", 11: "REGV", 12: "RCW16"}
+     9: "REGX", 10: "RCW", 11: "REGV", 12: "RCW16", 13: "RCWD", 14: "RCWP"}
 
 
 def main():
