@@ -346,7 +346,8 @@ def per_n_sweep(bsp, torch, dev, stream, ns, batch, chunk, reps=5, conv=True, co
     the event pair).  For n <= copy_ref_max_n a plain device copy of the same
     byte count is timed alongside (the small-n ceiling).  With ``conv`` the
     canonical path (canonical -> interleaved, factor, -> canonical) is timed
-    too (BASELINE configs[3])."""
+    too (BASELINE configs[3]), and for n <= CANON_MAX_N the fused canonical
+    call (batch_spotrf_canonical: conversion inside the factorization kernel)."""
     maxn = max(ns)
     A = torch.empty(bsp.batch_interleaved_elems(maxn, batch, chunk), dtype=torch.float32, device=dev)
     canon = torch.empty(batch * maxn * maxn, dtype=torch.float32, device=dev) if conv else None
@@ -417,6 +418,26 @@ def per_n_sweep(bsp, torch, dev, stream, ns, batch, chunk, reps=5, conv=True, co
             row["convert_in_gbs"] = round(cb / (mi * 1e-3) / 1e9, 1)
             row["convert_out_gbs"] = round(cb / (mo * 1e-3) / 1e9, 1)
             row["canonical_path_gflops"] = round(batch * flops_per_matrix(n) / ((mi + ms + mo) * 1e-3) / 1e9, 1)
+            if n <= bsp.CANON_MAX_N:
+                # the fused canonical call (batch_spotrf_canonical) on the same
+                # matrices in canonical storage: algorithmic bytes as above
+                fz = []
+                cnt.zero_()
+                for _ in range(reps):
+                    bsp.bspotrf_synth_generate(n, batch, chunk, Av, kind="dd", seed=2017, stream=stream)
+                    bsp.batch_interleaved_to_canonical(n, batch, chunk, Av, cv, stream=stream)
+                    bsp.bspotrf_fill_u32(flush, 0x3F800000, stream=stream)
+                    e0, e1 = Ev(), Ev()
+                    e0.record(stream)
+                    bsp.batch_spotrf_canonical(n, batch, cv, info, nfailed=cnt, stream=stream)
+                    e1.record(stream)
+                    fz.append((e0, e1))
+                torch.cuda.synchronize(dev)
+                if int(cnt.item()) != 0:
+                    raise SystemExit(f"bench per-n: {int(cnt.item())} canonical failures on SPD input at n={n}")
+                mf = median([x.elapsed_time(y) for x, y in fz])
+                row["canonical_fused_gbs"] = round(byt / (mf * 1e-3) / 1e9, 1)
+                row["canonical_fused_gflops"] = round(batch * flops_per_matrix(n) / (mf * 1e-3) / 1e9, 1)
         rows.append(row)
     del A, canon, flush
     torch.cuda.empty_cache()

@@ -218,6 +218,29 @@ int batch_interleaved_to_canonical(int n, int64_t batch, int chunk,
                                    float *dst_canonical,
                                    bspotrf_stream_t stream);
 
+/* ---- Canonical storage, conversion fused (round 2) -----
+ * The factorization on CANONICAL storage: A = batch consecutive n x n
+ * column-major matrices (lda = n), factored in place, lower,
+ * with the layout conversion fused into the kernel's loads and stores instead
+ * of canonical -> interleaved -> factor -> canonical (3 launches, 2 x 8n^2
+ * extra bytes per matrix).  A warp owns 32 consecutive matrices: each lane
+ * cp.asyncs its own lower triangle into a shared image (the 32 sectors of an
+ * instruction are re-hit in L1 by the next copies of the same column), the
+ * factorization is REG's (same per-element FP32 op sequence as every
+ * interleaved variant: bitwise the same L and info), and each final column is
+ * stored with a flat mapping (a warp store = 32 consecutive run elements).
+ *   n        1..BSPOTRF_CANON_MAX_N (20); n = 0 or batch = 0: quick return 0
+ *   A        device float*, batch*n*n floats, 4-B aligned; only lower-triangle
+ *            elements are read and written
+ *   info     device int32[batch], LAPACK convention (as the interleaved call)
+ *   nfailed  device int32* or NULL, incremented by the failure count
+ * Errors: -1 n, -2 batch, -3 A null/misaligned, -4 info null; positive =
+ * CUDA error.  Larger n: batch_canonical_to_interleaved + the interleaved
+ * call + batch_interleaved_to_canonical. */
+#define BSPOTRF_CANON_MAX_N 20
+int batch_spotrf_canonical(int n, int64_t batch, float *A, int32_t *info,
+                           int32_t *nfailed, bspotrf_stream_t stream);
+
 /* End-to-end call on HOST buffers (blocking).  hA is the interleaved storage
  * in host memory, hinfo host int32[batch], nfailed_out host int32* or NULL
  * (set, not incremented).  Only the lower triangles cross PCIe.

@@ -17,8 +17,8 @@ import threading
 __all__ = [
     "BspotrfError", "lib", "bspotrf_version", "batch_interleaved_elems",
     "batch_spotrf_interleaved", "batch_spotrf_interleaved_ex", "bspotrf_get_tuning",
-    "batch_canonical_to_interleaved", "batch_interleaved_to_canonical",
-    "batch_spotrf_interleaved_host", "batch_spotrf_host_bytes",
+    "batch_canonical_to_interleaved", "batch_interleaved_to_canonical", "batch_spotrf_canonical",
+    "CANON_MAX_N", "batch_spotrf_interleaved_host", "batch_spotrf_host_bytes",
     "bspotrf_synth_generate", "bspotrf_fill_u32", "bspotrf_probe_copy_lower", "Tuning",
     "batch_interleaved_rhs_elems", "batch_spotrs_interleaved", "batch_sposv_interleaved",
     "bspotrf_tuning_available", "VARIANT_AUTO", "VARIANT_REG", "VARIANT_SMEM", "VARIANT_TILE", "VARIANT_PANEL", "VARIANT_PTMEM", "VARIANT_RTMA", "VARIANT_RTMAP", "VARIANT_QTM", "VARIANT_REGX", "VARIANT_RCW", "VARIANT_REGV", "VARIANT_RCW16", "VARIANT_RCWD", "VARIANT_RCWP",
@@ -31,6 +31,7 @@ LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libbspotrf.
  VARIANT_RTMA, VARIANT_RTMAP, VARIANT_QTM, VARIANT_REGX, VARIANT_RCW, VARIANT_REGV, VARIANT_RCW16,
  VARIANT_RCWD, VARIANT_RCWP) = 0, 1, 2, 3, 4, 5, 6, 7, 8, 9, 10, 11, 12, 13, 14
 SYNTH_KINDS = {"dd": 0, "als": 1, "l0": 2}
+CANON_MAX_N = 20          # BSPOTRF_CANON_MAX_N
 UPPER_MODES = {"mirror": 0, "nan": 1, "keep": 2}
 
 # every exported symbol of include/*.h (checked by tests/test_abi.py)
@@ -40,7 +41,7 @@ EXPORTS = (
     "batch_interleaved_to_canonical", "batch_spotrf_interleaved_host", "batch_spotrf_host_bytes",
     "bspotrf_synth_generate", "bspotrf_fill_u32", "bspotrf_probe_copy_lower",
     "batch_interleaved_rhs_elems", "batch_spotrs_interleaved", "batch_sposv_interleaved",
-    "bspotrf_tuning_available",
+    "bspotrf_tuning_available", "batch_spotrf_canonical",
 )
 
 
@@ -74,6 +75,7 @@ _SIGS = {
     "bspotrf_tuning_available": (_i32, [_i32, _i32, ctypes.POINTER(Tuning)]),
     "batch_canonical_to_interleaved": (_i32, [_i32, _i64, _i32, _vp, _vp, _vp]),
     "batch_interleaved_to_canonical": (_i32, [_i32, _i64, _i32, _vp, _vp, _vp]),
+    "batch_spotrf_canonical": (_i32, [_i32, _i64, _vp, _vp, _vp, _vp]),
     "batch_spotrf_interleaved_host": (_i32, [_i32, _i64, _i32, _vp, _vp, _vp, _i64, _vp]),
     "batch_spotrf_host_bytes": (_i64, [_i32, _i64, _i32]),
     "bspotrf_synth_generate": (_i32, [_i32, _i64, _i32, _i64, _i32, _u64, _i32, _u64, _i64, _vp, _vp]),
@@ -207,6 +209,17 @@ def batch_interleaved_to_canonical(n, batch, chunk, src, dst, stream=None):
         _need(dst, batch * n * n, "torch.float32", "dst")
     return _check("batch_interleaved_to_canonical", lib().batch_interleaved_to_canonical(
         n, batch, chunk, _ptr(src), _ptr(dst), _stream(stream)))
+
+
+def batch_spotrf_canonical(n, batch, A, info, nfailed=None, stream=None):
+    """In-place batched SPOTRF (lower) on device CANONICAL storage A (batch
+    consecutive n x n column-major matrices), conversion fused; n <= CANON_MAX_N."""
+    if n and batch:
+        _need(A, batch * n * n, "torch.float32", "A")
+        _need(info, batch, "torch.int32", "info")
+        _need(nfailed, 1, "torch.int32", "nfailed")
+    return _check("batch_spotrf_canonical", lib().batch_spotrf_canonical(
+        n, batch, _ptr(A), _ptr(info), _ptr(nfailed), _stream(stream)))
 
 
 def batch_spotrf_interleaved_host(n, batch, chunk, hA, hinfo, slab=0, stream=None):

@@ -19,13 +19,16 @@ def main():
           f"dd generator; {pn.get('timing')}.  Fraction of the measured {peak} GB/s copy bandwidth "
           "(MEASURED_PEAKS.json).  Conversion: canonical <-> interleaved of the same batch "
           "(8 n^2 bytes per matrix per direction); canonical path = convert in + factor + convert out.\n")
-    print("| n | kernel | GB/s | frac | Gflop/s | vs copy | convert in GB/s (frac) | convert out GB/s (frac) | canonical path Gflop/s |")
-    print("|---|---|---|---|---|---|---|---|---|")
+    print("| n | kernel | GB/s | frac | Gflop/s | vs copy | convert in GB/s (frac) | convert out GB/s (frac) | "
+          "canonical path Gflop/s | fused canonical Gflop/s (GB/s) |")
+    print("|---|---|---|---|---|---|---|---|---|---|")
     for x in pn.get("rows", []):
         ci, co = x.get("convert_in_gbs"), x.get("convert_out_gbs")
         f = lambda v: f"{v:.0f} ({v / peak:.2f})" if v else "-"
         print(f"| {x['n']} | {V[x['variant']]} | {x['gbs']:.0f} | {x['frac']:.3f} | {x['gflops']:.0f} | "
-              f"{x.get('vs_copy', '-')} | {f(ci)} | {f(co)} | {x.get('canonical_path_gflops', '-')} |")
+              f"{x.get('vs_copy', '-')} | {f(ci)} | {f(co)} | {x.get('canonical_path_gflops', '-')} | "
+              + (f"{x['canonical_fused_gflops']:.0f} ({x['canonical_fused_gbs']:.0f})" if "canonical_fused_gbs" in x else "-")
+              + " |")
     if pl:
         print(f"\nn <= 4 at {pl.get('batch')} matrices (out of the launch-latency regime):\n")
         print("| n | kernel | GB/s | frac | vs copy | convert in GB/s (frac) | convert out GB/s (frac) |")

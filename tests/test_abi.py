@@ -76,6 +76,14 @@ def test_argument_errors_enqueue_nothing(L):
     assert h(4, 10, 32, None, fake, None, 0, None) == -4
     nf = ctypes.c_int32(99)
     assert h(0, 10, 32, None, None, ctypes.addressof(nf), 0, None) == 0 and nf.value == 0
+    c = L.batch_spotrf_canonical
+    assert c(-1, 10, fake, fake, None, None) == -1
+    assert c(21, 10, fake, fake, None, None) == -1       # BSPOTRF_CANON_MAX_N = 20
+    assert c(4, -1, fake, fake, None, None) == -2
+    assert c(4, 10, None, fake, None, None) == -3
+    assert c(4, 10, fake + 2, fake, None, None) == -3    # not 4-B aligned
+    assert c(4, 10, fake, None, None, None) == -4
+    assert c(0, 10, None, None, None, None) == 0 and c(4, 0, None, None, None, None) == 0
     s = L.bspotrf_synth_generate
     assert s(4, 10, 32, 0, 7, 1, 0, 0, 0, fake, None) == -5
     assert s(4, 10, 32, 0, 0, 1, 9, 0, 0, fake, None) == -6
