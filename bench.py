@@ -18,7 +18,7 @@ configs[2] (n=32, batch=4M per GPU, chunk 32, ALS-shaped), the largest
 single-GPU config -- weak scaling over GPUs.  The line also carries the "vs n"
 half of the metric ("per_n": every n in 1..64 at 1M matrices, the table's
 kernel, fraction of measured HBM bandwidth, the canonical path with layout
-conversion; "per_n_large_batch": n <= 4 at 64M matrices), measured after the
+conversion; "per_n_large_batch": n <= 8 at 64M matrices), measured after the
 timed region.
 
 Prints ONE JSON line (rank 0).  Metric unit: Gflop/s with n^3/3 flops per
@@ -94,7 +94,7 @@ def parse():
     ap.add_argument("--same-device", action="store_true",
                     help="test mode: every rank uses cuda:0 (needs --dist-backend gloo)")
     ap.add_argument("--per-n", default="1-64",
-                    help="n values of the per-n block (1M matrices, chunk 32; n <= 4 also at 64M), "
+                    help="n values of the per-n block (1M matrices, chunk 32; n <= 8 also at 64M), "
                          "e.g. 1-32,48,64, or none")
     return ap.parse_args()
 
@@ -580,10 +580,10 @@ def run_ours(a, w):
     if world == 1 and a.per_n != "none":
         ns = parse_ns(a.per_n)
         per_n = per_n_sweep(bsp, torch, dev, stream, ns, 1 << 20, 32, peak=peak, tag="1M")
-        small_ns = [x for x in ns if x <= 4]
+        small_ns = [x for x in ns if x <= 8]
         if small_ns:
             per_n_large = per_n_sweep(bsp, torch, dev, stream, small_ns, 1 << 26, 32, conv=True,
-                                      peak=peak, tag="64M (n <= 4 leave the launch-latency regime)")
+                                      peak=peak, tag="64M (n <= 8: out of the launch-latency regime)")
 
     cpu = None
     if rank == 0 and world == 1 and not a.no_cpu_baseline:

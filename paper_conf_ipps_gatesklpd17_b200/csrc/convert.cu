@@ -709,7 +709,8 @@ convert2d_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv2Shap
 //   carry      slots 8, 9 of row = lane.
 // Shared tile: row R starts at R*P + 4*t(R >> 2) (rows 16-B aligned, x =
 // 0..39 used); the per-row shift t and pitch P depend only on the class of E
-// mod 8 (odd n: 1, n = 2 mod 4: 4) and make the line side conflict-free (the 8
+// mod 8 (odd n: 1; n = 2 mod 4: 4, whose table also serves E = 0 mod 8) and
+// make the line side conflict-free (the 8
 // rows 4*l8 + j of one STS hit 8 disjoint 4-bank groups; found by exhaustive
 // search); the slot side reads one row's 8 contiguous slots per quarter warp.
 // All tile addresses are a per-lane base + a compile-time immediate.  (A first
@@ -979,8 +980,8 @@ cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float
             // 32-B aligned (E % 8 != 0) and rows span enough slices (odd n >= 13,
             // n = 2 mod 4 >= 10; below, the partial first / last sectors of the
             // few slices per row cost more than they save: profiles/r02/convert_v3.md)
-            const bool v3 = dir == 1 && E > 32 && E % 8 != 0 &&
-                            (ov == 3 || (ov == 0 && n >= (E % 8 == 1 ? 13 : 10)));
+            const bool v3 = dir == 1 && E > 32 &&
+                            (ov == 3 || (ov == 0 && E % 8 != 0 && n >= (E % 8 == 1 ? 13 : 10)));
             const cudaError_t e = v3 ? (E % 8 == 1 ? launch_v3<1>(n, G, C, src, dst, stream)
                                                    : launch_v3<4>(n, G, C, src, dst, stream))
                                      : (dir == 0 ? launch_v2<0>(n, G, C, src, dst, stream)
