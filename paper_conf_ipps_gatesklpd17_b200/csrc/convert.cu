@@ -26,8 +26,9 @@
 // between load and store phases) reached 2.4-2.9 TB/s (profiles/r01/c4_nsweep_r17.md).
 // Which kernel runs (launch_convert): v1 (below) for the ragged last group and
 // C % 4 != 0; v2 (128-bit both sides, paths A / B / D) for the full groups;
-// v3 (sector-aligned row streams) for interleaved -> canonical at E % 8 != 0,
-// n >= 13 (profiles/r02/convert_v3.md).
+// for interleaved -> canonical, v4 (whole-group image, one bulk store) at
+// E % 8 != 0, n = 7..30 and v3 (sector-aligned row streams) at odd n >= 31,
+// n = 2 mod 4 >= 34 and n = 4 mod 8 >= 28 (profiles/r02/convert_v3.md).
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <stdlib.h>
@@ -854,6 +855,105 @@ convert3_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv3Shape
     }
 }
 
+// ---- v4: interleaved -> canonical at odd n, a whole-group image + ONE bulk store
+// The canonical block of a 32-matrix group is 32*E contiguous floats (128*E
+// bytes, 16-B aligned for any E).  A CTA loads the group's E interleaved lines
+// (256 threads, two 32-line steps per warp in flight), puts them into a shared
+// image of that block (row m = matrix at m*E; for odd E the 32 lanes of one STS
+// hit 32 distinct banks: 4*l8*E mod 32 takes 8 distinct multiples of 4) and one
+// thread writes the image with a single cp.async.bulk shared -> global: every
+// sector of the canonical side is written whole, once, by the copy engine.  Two
+// images (when they fit) let group g+1 load while group g's store drains.
+__device__ __forceinline__ uint32_t cv4_smem_u32(const void *p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void cv4_bulk_s2g(void *dst, const void *src, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst),
+                 "r"(cv4_smem_u32(src)), "r"(bytes)
+                 : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+template <int K>
+__device__ __forceinline__ void cv4_bulk_wait_read() {      // <= K bulk groups may still read smem
+    asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(K) : "memory");
+}
+
+struct Cv4Shape {
+    int64_t C, G;
+    int E, WPG;            // warps per group (1, 2, 4, 8): ceil(E / 64) rounded up; 8 / WPG groups per CTA step
+};
+
+template <int NB>
+__global__ void __launch_bounds__(CV_THREADS, 2)
+convert4_kernel(const float *__restrict__ src, float *__restrict__ dst, Cv4Shape s) {
+    extern __shared__ __align__(128) float cv4_smem[];
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const int E = s.E, WPG = s.WPG, GP = CV_WARPS / WPG;
+    const int gi = w / WPG, wg = w - gi * WPG;            // group slot of this warp, warp within the group
+    const bool leader = wg == 0 && lane == 0;             // issues (and waits for) the slot's bulk stores
+    const int l8 = lane & 7, lq = lane >> 3, c4 = 4 * l8;
+    const int step = 32 * WPG;                            // lines per group step
+    int it = 0;
+    for (int64_t g0 = (int64_t)blockIdx.x * GP; g0 < s.G; g0 += (int64_t)gridDim.x * GP, ++it) {
+        const int64_t g = g0 + gi;
+        float *img = cv4_smem + ((size_t)gi * NB + (NB == 1 ? 0 : (it & 1))) * 32 * E;
+        if (leader) cv4_bulk_wait_read<NB - 1>();         // the store issued from this image has read it
+        __syncthreads();
+        if (g < s.G) {
+            const int64_t m0 = g * 32;
+            const float *lb = src + (m0 / s.C) * s.C * (int64_t)E + m0 % s.C + c4;
+            float *r0 = img + c4 * E;                      // row 4*l8 (+ j*E for rows 4*l8 + j)
+            for (int base = 32 * wg + lq; base < E; base += 2 * step) {
+                float4 R[16];
+#pragma unroll
+                for (int kk = 0; kk < 16; ++kk) {
+                    const int line = base + (kk >> 3) * step + 4 * (kk & 7);
+                    if (line < E) R[kk] = ldg4(lb + (int64_t)line * s.C);
+                }
+#pragma unroll
+                for (int kk = 0; kk < 16; ++kk) {
+                    const int line = base + (kk >> 3) * step + 4 * (kk & 7);
+                    if (line < E) {
+                        r0[line] = R[kk].x;
+                        r0[E + line] = R[kk].y;
+                        r0[2 * E + line] = R[kk].z;
+                        r0[3 * E + line] = R[kk].w;
+                    }
+                }
+            }
+        }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic STS -> async-proxy read
+        __syncthreads();
+        if (leader && g < s.G) cv4_bulk_s2g(dst + g * 32 * (int64_t)E, img, (uint32_t)(128 * E));
+    }
+    if (leader) cv4_bulk_wait_read<0>();                  // the images outlive the last stores' reads
+}
+
+static cudaError_t launch_v4(int n, int64_t G, int64_t C, const float *src, float *dst, cudaStream_t stream) {
+    Cv4Shape s;
+    s.C = C;
+    s.G = G;
+    s.E = n * n;
+    const int wpg = (s.E + 63) / 64;                      // a warp covers 64 lines per pass (two 32-line steps)
+    s.WPG = wpg <= 1 ? 1 : (wpg <= 2 ? 2 : (wpg <= 4 ? 4 : 8));
+    const size_t img = (size_t)128 * s.E * (CV_WARPS / s.WPG);   // one image per group slot
+    const bool two = 2 * img <= (size_t)113 * 1024;
+    const size_t smem = two ? 2 * img : img;
+    auto kern = two ? convert4_kernel<2> : convert4_kernel<1>;
+    int dev = 0, sms = 148, per_sm = 1;
+    if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, CV_THREADS, smem);
+    if (per_sm < 1) per_sm = 1;
+    const int gp = CV_WARPS / s.WPG;
+    int64_t grid = (int64_t)sms * per_sm;
+    const int64_t need = (G + gp - 1) / gp;
+    if (grid > need) grid = need;
+    kern<<<(unsigned)grid, CV_THREADS, smem, stream>>>(src, dst, s);
+    return cudaGetLastError();
+}
+
 template <typename K>
 static cudaError_t launch_persistent(K kern, int64_t tiles, const float *src, float *dst, const Cv2Shape &s,
                                      cudaStream_t stream, size_t dyn_smem = 0) {
@@ -954,11 +1054,11 @@ static cudaError_t launch_v3(int n, int64_t G, int64_t C, const float *src, floa
 }
 
 // v3 (fixed slices, constant phases) vs v2, per direction and n: see the
-// choice in launch_convert.  BSPOTRF_CONVERT_PATH=v2|v3 forces one (probes).
+// choice in launch_convert.  BSPOTRF_CONVERT_PATH=v2|v3|v4 forces one (probes).
 static int convert_path_override() {
     const char *v = getenv("BSPOTRF_CONVERT_PATH");
-    if (!v) return 0;
-    return (v[0] == 'v' && v[1] == '3') ? 3 : ((v[0] == 'v' && v[1] == '2') ? 2 : 0);
+    if (!v || v[0] != 'v') return 0;
+    return v[1] == '4' ? 4 : (v[1] == '3' ? 3 : (v[1] == '2' ? 2 : 0));
 }
 
 cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float *src, float *dst,
@@ -976,13 +1076,19 @@ cudaError_t launch_convert(int dir, int n, int64_t batch, int64_t C, const float
         if (G > 0) {
             const int ov = convert_path_override();
             const int E = n * n;
-            // interleaved -> canonical: v3 where v2's canonical rows are not
-            // 32-B aligned (E % 8 != 0) and rows span enough slices (odd n >= 13,
-            // n = 2 mod 4 >= 10; below, the partial first / last sectors of the
-            // few slices per row cost more than they save: profiles/r02/convert_v3.md)
-            const bool v3 = dir == 1 && E > 32 &&
-                            (ov == 3 || (ov == 0 && E % 8 != 0 && n >= (E % 8 == 1 ? 13 : 10)));
-            const cudaError_t e = v3 ? (E % 8 == 1 ? launch_v3<1>(n, G, C, src, dst, stream)
+            // interleaved -> canonical, per n class (profiles/r02/convert_v3.md, j19/j19b A/B):
+            //   n = 7..30, E % 8 != 0  v4 (whole-group image, one bulk store per group)
+            //   odd n >= 31         v3 (the image no longer leaves room for two per SM)
+            //   n = 2 mod 4, >= 34  v3 (v2's odd rows start mid-sector)
+            //   n = 4 mod 8, >= 28  v3 (rows 64-B but not 128-B aligned: v2 0.71-0.76)
+            //   otherwise           v2
+            const bool odd = E % 2 == 1;
+            const bool def4 = E % 8 != 0 && n >= 7 && n <= 30;
+            const bool def3 = (odd && n >= 31) || (E % 8 == 4 && n >= 10) || (E % 32 == 16 && n >= 28);
+            const bool v4 = dir == 1 && E >= 36 && E <= 961 && E % 32 != 0 && (ov == 4 || (ov == 0 && def4));
+            const bool v3 = dir == 1 && !v4 && E > 32 && (ov == 3 || (ov == 0 && def3));
+            const cudaError_t e = v4 ? launch_v4(n, G, C, src, dst, stream) :
+                                  v3 ? (E % 8 == 1 ? launch_v3<1>(n, G, C, src, dst, stream)
                                                    : launch_v3<4>(n, G, C, src, dst, stream))
                                      : (dir == 0 ? launch_v2<0>(n, G, C, src, dst, stream)
                                                  : launch_v2<1>(n, G, C, src, dst, stream));

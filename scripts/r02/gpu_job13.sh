@@ -12,7 +12,7 @@ ctests)
   timeout 1200 python -m pytest tests/test_gpu_layout_synth_host.py -m gpu -q -p no:cacheprovider -x -k "conversion" > $O/pytest_conv.log 2>&1; echo "ctests rc=$?"
   tail -n 15 $O/pytest_conv.log ;;
 ab)
-  timeout 1200 python scripts/r02/conv_ab.py ${AB_N:-6-64} v2,v3 > $O/conv_ab.jsonl 2> $O/conv_ab.err; echo "ab rc=$?"; tail -3 $O/conv_ab.err ;;
+  timeout 1200 python scripts/r02/conv_ab.py ${AB_N:-6-64} ${AB_P:-v2,v3} > $O/conv_ab.jsonl 2> $O/conv_ab.err; echo "ab rc=$?"; tail -3 $O/conv_ab.err ;;
 ptests)
   timeout 1800 python -m pytest tests -m gpu -q -p no:cacheprovider -x -k "rcw or c4 or table or default" > $O/pytest_p.log 2>&1; echo "ptests rc=$?"
   tail -n 3 $O/pytest_p.log ;;

@@ -53,11 +53,12 @@ def _roundtrip_exact(n, batch, chunk, seed):
     assert np.array_equal(back.cpu().numpy().view(np.uint32), canon.reshape(-1).view(np.uint32))
 
 
-@pytest.mark.parametrize("path", ["v3", "v2"])
+@pytest.mark.parametrize("path", ["v4", "v3", "v2"])
 @pytest.mark.parametrize("n", [6, 7, 10, 11, 12, 14, 17, 18, 30, 33, 34, 50, 61, 62, 64])
 @pytest.mark.parametrize("chunk,batch", [(32, 1184), (0, 9632), (96, 4096 + 32 * 7 + 5)])
 def test_conversion_paths_forced(monkeypatch, path, n, chunk, batch):
-    """v3 (fixed 32-element slices, per-lane constant row phases, carries between
+    """v4 (odd n: whole-group image + one bulk store), v3 (fixed 32-element
+    slices, per-lane constant row phases, carries between
     slices) and v2 (proportional / aligned slices), each forced on every n
     class -- E % 4 in {0, 1}, E % 8 in {0, 4}, the last slice 1..32 wide -- with
     small group counts, where every group is cut into many segments (a unit =
