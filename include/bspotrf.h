@@ -207,7 +207,11 @@ int bspotrf_get_tuning(int n, int chunk, bspotrf_tuning *out);
 /* Layout conversion, out of place, bit-exact (a pure permutation):
  * canonical = batch consecutive n x n column-major matrices,
  * batch*n*n floats; interleaved as above.  src and dst must not overlap.
- * Pad lanes of the interleaved side are never read or written.
+ * Pad lanes of the interleaved side are never read or written.  The kernel
+ * is chosen per direction and n class (v1 / v2 / v3 / v4); the
+ * environment variable BSPOTRF_CONVERT_PATH=v2|v3|v4, read per call, forces
+ * one where it applies (an A/B probe for the benchmarks; every path produces
+ * the same bits, tested).
  * Errors: -1 n, -2 batch, -3 chunk, -4 src null, -5 dst null or overlapping. */
 int batch_canonical_to_interleaved(int n, int64_t batch, int chunk,
                                    const float *src_canonical,
