@@ -80,8 +80,8 @@ def main():
             want = [n, 32 if c == 32 else 0, e["param"]]
         elif v in (12, 13):
             want = [n, 32 if c == 32 else 0]
-        elif v == 14:                             # <N, CT, D1>
-            want = [n, 32 if c == 32 else 0, e["param"]]
+        elif v == 14:                             # <N, CT, D1, TM>: runtime chunks staged by 2-D TMA
+            want = [n, 32, e["param"], 0] if c == 32 else [n, 0, e["param"], 1]
         elif v == 9:
             want = [n, e["param"], e["staging"]]
         elif v in (6, 7, 3):

@@ -136,6 +136,31 @@ def test_rcw_parity_failures_ragged(n, chunk):
         assert_parity(n, batch, chunk, canon, inter, out, info, cnt)
 
 
+@pytest.mark.parametrize("n", [33, 49, 57, 64])
+@pytest.mark.parametrize("chunk,batch", [(0, 5 * 32 + 12), (0, 4 * 2 * 148 * 32 + 44), (64, 5 * 32 + 12),
+                                         (160, 3 * 160 + 37)])
+def test_rcwp_tma2d_runtime_chunk(n, chunk, batch):
+    """RCWP at runtime chunks whose stride is a multiple of 16 B stages each
+    column block by 2-D TMA boxes (32 matrices x (N - 8c) rows) from one tensor
+    map per block: against the oracle and bitwise against RCW, with failures, a
+    partial last group (chunk 0: the box runs past the row end and is
+    zero-filled; other chunks: pad lanes) and, at the large batch, several
+    groups per persistent CTA."""
+    canon, inter = make_batch(n, batch, chunk, kind="dd", seed=n + 3, fail_seed=2018, fail_period=7)
+    failed, kk = synth.fail_plan(n, 2018, 7, np.arange(batch, dtype=np.uint64))
+    ref = None
+    for t in [dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0) for d1 in (0, 1)] + \
+             [dict(variant=bsp.VARIANT_RCW, threads_per_block=256, param=_rcw_ncta(n)[0], staging=0)]:
+        out, info, cnt = run_gpu(n, batch, chunk, inter, tune=t)
+        assert np.array_equal(info, np.where(failed, kk + 1, 0)), t
+        if ref is None:
+            if batch < 10000:
+                assert_parity(n, batch, chunk, canon, inter, out, info, cnt)
+            ref = out
+        else:
+            assert np.array_equal(out.view(np.uint32), ref.view(np.uint32)), t
+
+
 @pytest.mark.parametrize("n", [36, 48, 52, 64])
 def test_rcw_integer_and_als(n):
     """RCW on the exactness set (P2: returns exactly L0) and on ALS-shaped input."""
