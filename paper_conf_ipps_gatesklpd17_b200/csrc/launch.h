@@ -96,7 +96,7 @@ cudaError_t launch_rcwd(const FactorArgs &a);
 
 // Variant RCWP: RCW with the factor in recycled TMEM pages, two CTAs per SM
 // (csrc/potrf_rcwp.cuh); D1: the diagonal block factored by one warp.
-template <int N, int CT, bool D1>
+template <int N, int CT, int P>
 cudaError_t launch_rcwp(const FactorArgs &a);
 
 // Variant TILE: the paper's top-looking tile algorithm, NB x NB register

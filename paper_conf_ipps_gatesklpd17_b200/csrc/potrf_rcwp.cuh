@@ -126,13 +126,13 @@ struct RcwpPages {
     }
 };
 
-template <int N>
+template <int N, int NC = 2>
 struct RcwpShape {
     static constexpr int R = (N + 7) / 8;
     static constexpr int UNIT = 8 * 8 * 32;              // floats per 8 KB unit
     static constexpr RcwpPages<R> PG{};
-    static constexpr int COLS = 256;                     // TMEM columns per CTA (two CTAs per SM)
-    static constexpr int WCOLS = 128;                    // per warp (warps h, h+4 share a lane quarter)
+    static constexpr int COLS = NC == 3 ? 128 : 256;     // TMEM columns per CTA (NC CTAs per SM)
+    static constexpr int WCOLS = COLS / 2;               // per warp (warps h, h+4 share a lane quarter)
     static constexpr size_t SMEM = (size_t)(R * UNIT + 44 * 32) * sizeof(float);
     static_assert(PG.valid(), "page colouring: live pages collide or exceed the bound");
     static_assert(PG.npages * 8 <= WCOLS, "live pages exceed the warp's TMEM columns");
@@ -144,11 +144,11 @@ struct RcwpShape {
 // reciprocals through shared memory, one more block barrier) instead of
 // redundantly by all eight warps -- ~250 instructions per warp and block fewer;
 // the idle warps' issue slots go to the SM's other CTA.
-template <int N, int CT, bool D1, bool TM>
-__global__ void __launch_bounds__(256, 2)
+template <int N, int CT, bool D1, bool TM, int NC>
+__global__ void __launch_bounds__(256, NC)
 potrf_rcwp_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__restrict__ nfailed,
                   int64_t batch, int64_t cs, const __grid_constant__ RcwpMaps maps) {
-    using SH = RcwpShape<N>;
+    using SH = RcwpShape<N, NC>;
     using RS = RcwShape<N, 1>;                           // stage geometry (rs, bytes, dt)
     constexpr int R = SH::R, UNIT = SH::UNIT;
     constexpr bool TMA = CT == 32;                       // one chunk == one group of 32
@@ -476,15 +476,16 @@ inline bool rcwp_make_maps(const FactorArgs &a, RcwpMaps *mp) {
     return true;
 }
 
-template <int N, int CT, bool D1, bool TM>
+template <int N, int CT, bool D1, bool TM, int NC>
 cudaError_t launch_rcwp_k(const FactorArgs &a, const RcwpMaps &maps) {
-    using SH = RcwpShape<N>;
-    auto kern = potrf_rcwp_kernel<N, CT, D1, TM>;
-    // two CTAs per SM own all 512 TMEM columns (256 each): ask for enough shared
-    // memory that a third CTA never becomes resident (it would spin in
-    // tcgen05.alloc until one of the two exits)
+    using SH = RcwpShape<N, NC>;
+    auto kern = potrf_rcwp_kernel<N, CT, D1, TM, NC>;
+    // NC CTAs per SM own NC * COLS <= 512 TMEM columns: ask for enough shared
+    // memory that CTA NC+1 never becomes resident (it would spin in
+    // tcgen05.alloc until another exits): 80 KB for two, 57 KB for three
     size_t sm = SH::SMEM;
-    if (sm < (size_t)80 * 1024) sm = (size_t)80 * 1024;
+    const size_t floor_sm = NC == 3 ? (size_t)57 * 1024 : (size_t)80 * 1024;
+    if (sm < floor_sm) sm = floor_sm;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
     if (const cudaError_t ce = apply_carveout(kern, a.carveout); ce != cudaSuccess) return ce;
@@ -493,21 +494,25 @@ cudaError_t launch_rcwp_k(const FactorArgs &a, const RcwpMaps &maps) {
     if (e == cudaSuccess) e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     if (e != cudaSuccess) return e;
     const int64_t groups = (a.batch + 31) / 32;
-    const int64_t grid = groups < (int64_t)nsm * 2 ? groups : (int64_t)nsm * 2;
+    const int64_t grid = groups < (int64_t)nsm * NC ? groups : (int64_t)nsm * NC;
     kern<<<(unsigned)grid, 256, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride, maps);
     return cudaGetLastError();
 }
 
-template <int N, int CT, bool D1>
+// P (the tuning param): bit 0 = D1, bit 1 = three CTAs per SM (128 TMEM columns
+// and <= 80 registers each; n <= 40, where a warp's live pages fit 64 columns).
+template <int N, int CT, int P>
 cudaError_t launch_rcwp(const FactorArgs &a) {
+    constexpr bool D1 = (P & 1) != 0;
+    constexpr int NC = (P & 2) ? 3 : 2;
     RcwpMaps maps{};
     // 2-D TMA staging where it measured faster than the per-thread cp.async form:
     // n <= 51 (+5-20% at runtime chunks, j24b); at n >= 52 the boxes of up to 64
     // rows of 128 B at a large stride are 2-15% slower.
     if constexpr (CT == 0 && N <= 51) {
-        if (rcwp_make_maps<N>(a, &maps)) return launch_rcwp_k<N, CT, D1, true>(a, maps);
+        if (rcwp_make_maps<N>(a, &maps)) return launch_rcwp_k<N, CT, D1, true, NC>(a, maps);
     }
-    return launch_rcwp_k<N, CT, D1, false>(a, maps);
+    return launch_rcwp_k<N, CT, D1, false, NC>(a, maps);
 }
 
 }  // namespace bsp

@@ -124,8 +124,8 @@ def candidates(n, chunk):
     if n in gen_instances.RCWD_N:
         c.append(dict(variant=bsp.VARIANT_RCWD, threads_per_block=288, param=0, staging=0))
     if n in gen_instances.RCWP_N:
-        for d1 in (0, 1):
-            c.append(dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0))
+        for prm in gen_instances.rcwp_params(n):
+            c.append(dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=prm, staging=0))
     for nb in (2, 4, 8):
         if nb <= n or nb == 2:
             for tpb in (64, 128, 256):

@@ -80,8 +80,9 @@ def main():
             want = [n, 32 if c == 32 else 0, e["param"]]
         elif v in (12, 13):
             want = [n, 32 if c == 32 else 0]
-        elif v == 14:                             # <N, CT, D1, TM>: runtime chunks staged by 2-D TMA
-            want = [n, 32, e["param"], 0] if c == 32 else [n, 0, e["param"], 1 if n <= 51 else 0]
+        elif v == 14:                             # <N, CT, D1, TM, NC>: runtime chunks staged by 2-D TMA
+            d1, nc = e["param"] & 1, 3 if e["param"] & 2 else 2
+            want = [n, 32, d1, 0, nc] if c == 32 else [n, 0, d1, 1 if n <= 51 else 0, nc]
         elif v == 9:
             want = [n, e["param"], e["staging"]]
         elif v in (6, 7, 3):

@@ -54,6 +54,12 @@ RCW_N = range(33, 65)
 RCW16_N = range(49, 65)
 RCWD_N = range(49, 65)
 RCWP_N = range(33, 65)
+
+
+def rcwp_params(n):
+    """RCWP tuning params: bit 0 = single-warp diagonal factorization, bit 1 =
+    three CTAs per SM (n <= 40: the live TMEM pages of a warp fit 64 columns)."""
+    return (0, 1, 2) if n <= 40 else (0, 1)
 RCW_CT = (32, 0)
 
 
@@ -334,11 +340,10 @@ def main():
         files.add(name)
     for n in RCWP_N:
         body = [hdr, '#include "../potrf_rcwp.cuh"', "namespace bsp {"]
-        for d1 in (0, 1):
+        for prm in rcwp_params(n):
             for ct in RCW_CT:
-                b = "true" if d1 else "false"
-                body.append(f"template cudaError_t launch_rcwp<{n}, {ct}, {b}>(const FactorArgs &);")
-                entries.append(f"{{14, {n}, {d1}, {ct}, 0, &launch_rcwp<{n}, {ct}, {b}>}}")
+                body.append(f"template cudaError_t launch_rcwp<{n}, {ct}, {prm}>(const FactorArgs &);")
+                entries.append(f"{{14, {n}, {prm}, {ct}, 0, &launch_rcwp<{n}, {ct}, {prm}>}}")
         body.append("}  // namespace bsp\n")
         name = f"inst_rcwp_{n:02d}.cu"
         write_if_changed(os.path.join(GEN, name), "\n".join(body))

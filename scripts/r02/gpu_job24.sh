@@ -11,5 +11,5 @@ rtests)
   timeout 1500 python -m pytest tests -m gpu -q -p no:cacheprovider -x -k "rcw or bitwise or variants" > $O/pytest_rcw.log 2>&1; echo "rtests rc=$?"
   tail -n 2 $O/pytest_rcw.log ;;
 sweep)
-  timeout 1500 python scripts/autotune.py --n 33-64 --chunks 0,64,128,256 --reps 5 --variants 10,14 --out $O/sweep.jsonl > $O/sweep.log 2>&1; echo "sweep rc=$?" ;;
+  timeout 1500 python scripts/autotune.py --n ${SW_N:-33-64} --chunks ${SW_C:-0,64,128,256} --reps 5 --variants ${SW_V:-10,14} --out $O/sweep.jsonl > $O/sweep.log 2>&1; echo "sweep rc=$?" ;;
 esac; done

@@ -129,7 +129,8 @@ def test_rcw_parity_failures_ragged(n, chunk):
     if n in gen_instances_mod().RCWD_N:
         ts.append(dict(variant=bsp.VARIANT_RCWD, threads_per_block=288, param=0, staging=0))
     if n in gen_instances_mod().RCWP_N:
-        ts += [dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0) for d1 in (0, 1)]
+        ts += [dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0)
+               for d1 in gen_instances_mod().rcwp_params(n)]
     for t in ts:
         out, info, cnt = run_gpu(n, batch, chunk, inter, tune=t)
         assert np.array_equal(info, np.where(failed, kk + 1, 0)), t
@@ -149,7 +150,8 @@ def test_rcwp_tma2d_runtime_chunk(n, chunk, batch):
     canon, inter = make_batch(n, batch, chunk, kind="dd", seed=n + 3, fail_seed=2018, fail_period=7)
     failed, kk = synth.fail_plan(n, 2018, 7, np.arange(batch, dtype=np.uint64))
     ref = None
-    for t in [dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0) for d1 in (0, 1)] + \
+    for t in [dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0)
+               for d1 in gen_instances_mod().rcwp_params(n)] + \
              [dict(variant=bsp.VARIANT_RCW, threads_per_block=256, param=_rcw_ncta(n)[0], staging=0)]:
         out, info, cnt = run_gpu(n, batch, chunk, inter, tune=t)
         assert np.array_equal(info, np.where(failed, kk + 1, 0)), t
@@ -246,7 +248,8 @@ def _tunings(n, chunk):
     if n in gen_instances_mod().RCWD_N:
         out.append(dict(variant=bsp.VARIANT_RCWD, threads_per_block=288, param=0, staging=0))
     if n in gen_instances_mod().RCWP_N:
-        out += [dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0) for d1 in (0, 1)]
+        out += [dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0)
+               for d1 in gen_instances_mod().rcwp_params(n)]
     if n <= 8:
         out.append(dict(variant=bsp.VARIANT_REGV, threads_per_block=128, param=0, staging=0))
     for tpb in (64, 256):
@@ -339,7 +342,8 @@ def test_rcw_many_groups_per_cta(n, chunk):
     if n in gen_instances_mod().RCWD_N:
         ts.append(dict(variant=bsp.VARIANT_RCWD, threads_per_block=288, param=0, staging=0))
     if n in gen_instances_mod().RCWP_N:
-        ts += [dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0) for d1 in (0, 1)]
+        ts += [dict(variant=bsp.VARIANT_RCWP, threads_per_block=256, param=d1, staging=0)
+               for d1 in gen_instances_mod().rcwp_params(n)]
     idx = np.unique(np.concatenate([np.arange(0, batch, 37), np.arange(batch - 200, batch),
                                     np.arange(0, 64 * 32, 31)]))
     ref = None
