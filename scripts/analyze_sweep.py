@@ -68,7 +68,7 @@ def main():
           f"correlation r = {corr:.4f} (the paper's Fig. 21).\n")
     print("| Parameter | %IncMSE (permutation, held-out 25%) | Type |")
     print("|---|---|---|")
-    types = ["integer", "categorical (12)", "binary", "integer", "integer", "integer", "categorical (3)",
+    types = ["integer", "categorical (14)", "binary", "integer", "integer", "integer", "categorical (3)",
              "integer (0 = default, 1..100 %)"]
     for f, v, t in sorted(zip(feats, imp, types), key=lambda x: -x[1]):
         print(f"| {f} | {v:.1f} | {t} |")
