@@ -188,6 +188,12 @@ int64_t batch_interleaved_elems(int n, int64_t batch, int chunk);
 int batch_spotrf_interleaved(int n, int64_t batch, int chunk, float *A,
                              int32_t *info, bspotrf_stream_t stream);
 
+/* Runtime chunks (any chunk but 32, including 0) whose stride is a multiple of
+ * 16 B stage some kernels' column runs by 2-D tensor TMA (RCWP n <= 51, PTMEM
+ * n = 32..38); the environment variable BSPOTRF_TMA2D=0, read per
+ * call, selects the per-thread cp.async staging instead (an A/B probe; the
+ * results are bitwise the same, tested). */
+
 /* As above, plus:
  *   nfailed  device int32* or NULL: atomically INCREMENTED by the number of
  *            matrices with info != 0 (the caller zeroes it) -- fused into the

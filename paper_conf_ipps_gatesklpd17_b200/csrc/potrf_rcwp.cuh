@@ -40,9 +40,7 @@
 #include "ptx.cuh"
 #include "potrf_rcw.cuh"
 #include "potrf_tmem.cuh"
-
-#include <cuda.h>
-#include <cudaTypedefs.h>
+#include "tma2d.cuh"
 
 namespace bsp {
 
@@ -55,14 +53,6 @@ namespace bsp {
 struct RcwpMaps {
     CUtensorMap m[8];
 };
-
-__device__ __forceinline__ void tma_load_2d(void *dst, const CUtensorMap *map, int x, int y, uint64_t *bar) {
-    asm volatile(
-        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
-            smem_u32(dst)),
-        "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar))
-        : "memory");
-}
 
 __device__ __forceinline__ void tmem_ld8(uint32_t taddr, float *v) {
     asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
@@ -436,20 +426,6 @@ potrf_rcwp_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__
     }
 }
 
-// cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda
-// link dependency); resolved once.
-inline PFN_cuTensorMapEncodeTiled_v12000 rcwp_encode_fn() {
-    static PFN_cuTensorMapEncodeTiled_v12000 fn = []() -> PFN_cuTensorMapEncodeTiled_v12000 {
-        void *p = nullptr;
-        cudaDriverEntryPointQueryResult q;
-        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
-            q != cudaDriverEntryPointSuccess)
-            return nullptr;
-        return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
-    }();
-    return fn;
-}
-
 // One map per column block c: the array as [rows][C] floats (rows = chunks * N^2,
 // row stride C*4 B), box 32 x (N - 8c).  False if the layout does not qualify
 // (C % 4 != 0 or C < 32: TMA needs 16-B strides and a box within the inner
@@ -457,22 +433,8 @@ inline PFN_cuTensorMapEncodeTiled_v12000 rcwp_encode_fn() {
 template <int N>
 inline bool rcwp_make_maps(const FactorArgs &a, RcwpMaps *mp) {
     constexpr int R = (N + 7) / 8;
-    const int64_t C = a.cstride;
-    if (C % 4 != 0 || C < 32) return false;
-    const int64_t rows = (a.batch + C - 1) / C * (int64_t)(N * N);
-    if (rows >= ((int64_t)1 << 31) || C >= ((int64_t)1 << 31)) return false;
-    auto enc = rcwp_encode_fn();
-    if (enc == nullptr) return false;
-    for (int c = 0; c < R; ++c) {
-        const cuuint64_t dims[2] = {(cuuint64_t)C, (cuuint64_t)rows};
-        const cuuint64_t strides[1] = {(cuuint64_t)C * 4};
-        const cuuint32_t box[2] = {32u, (cuuint32_t)(N - 8 * c)};
-        const cuuint32_t estr[2] = {1u, 1u};
-        if (enc(&mp->m[c], CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, a.A, dims, strides, box, estr,
-                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
-            return false;
-    }
+    for (int c = 0; c < R; ++c)
+        if (!tma2d_make_map(&mp->m[c], a.A, a.batch, a.cstride, N * N, N - 8 * c)) return false;
     return true;
 }
 

@@ -26,6 +26,7 @@
 #include "launch.h"
 #include "potrs.cuh"
 #include "ptx.cuh"
+#include "tma2d.cuh"
 
 namespace bsp {
 
@@ -99,6 +100,15 @@ struct TmemShape {
     static_assert(CTM >= 1, "TMEM must hold at least one tile column");
 };
 
+// Runtime-chunk staging of the shared-memory panel columns CS..S-1 by 2-D TMA
+// (round 2, tma2d.cuh): one box of 32 matrices x (N - c) rows per column c,
+// one tensor map per column (its box height).
+template <int K>
+struct PtmemMaps {
+    CUtensorMap m[K > 0 ? K : 1];
+};
+
+
 // SOLVE: fused SPOSV with one right-hand side: B (n x 1 per
 // matrix, interleaved like A) is solved while every column of L is still on
 // chip -- forward substitution rides along the panel tile loop and the
@@ -108,10 +118,11 @@ struct TmemShape {
 // FILLT: TMEM tiles loaded per warp-synchronised batch of the fill (0 = the
 // default: 5 with TMA staging, 1 with per-thread cp.async); a tuning axis
 // (bspotrf_tuning.staging 3 = TMA with 12), see the fill below.
-template <int N, int CT, int S, bool TMA, bool SOLVE = false, int FILLT = 0>
+template <int N, int CT, int S, bool TMA, bool SOLVE = false, int FILLT = 0, bool TM = false>
 __global__ void __launch_bounds__(128, TmemShape<N, S>::COLS == 256 ? 2 : 1)
 potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                    int32_t *__restrict__ nfailed, int64_t batch, int64_t cs,
+                   const __grid_constant__ PtmemMaps<S - TmemShape<N, S>::CS> maps,
                    float *__restrict__ Bx = nullptr) {
     using SH = TmemShape<N, S>;
     constexpr int NB = 4, TR = SH::TR, TC = SH::TC, CTM = SH::CTM, CS = SH::CS;
@@ -138,7 +149,7 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
         tmem_alloc(&tmem_base_sh, SH::COLS);
         tmem_relinquish();
     }
-    if constexpr (TMA && PSM > 0) {
+    if constexpr ((TMA || TM) && PSM > 0) {
         if (lane == 0) {
             mbar_init(&bars[warp], 1);
             mbar_fence_init();
@@ -163,6 +174,17 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                 for (int c = CS; c < S; ++c)
                     bulk_g2s(smem + (size_t)warp * QW * 32 + qs(c, c) * 32, chunk + (c + c * N) * 32,
                              (uint32_t)((N - c) * 32 * 4), &bars[warp]);
+            }
+        } else if constexpr (TM) {
+            if (lane == 0) {
+                int64_t m0 = (int64_t)blockIdx.x * 128 + warp * 32;
+                if (m0 >= batch) m0 = (batch - 1) / 32 * 32;   // idle warp past the end: a valid group
+                const int x = (int)(m0 % cs), y = (int)((m0 / cs) * (int64_t)(N * N));
+                mbar_arrive_expect_tx(&bars[warp], (uint32_t)(PSM * 32 * 4));
+#pragma unroll 1
+                for (int c = CS; c < S; ++c)
+                    tma_load_2d(smem + (size_t)warp * QW * 32 + qs(c, c) * 32, &maps.m[c - CS], x, y + c + c * N,
+                                &bars[warp]);
             }
         } else {
 #pragma unroll 1
@@ -217,7 +239,7 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
     });
     tmem_wait_st();
     if constexpr (PSM > 0) {
-        if constexpr (TMA) mbar_wait(&bars[warp], 0);
+        if constexpr (TMA || TM) mbar_wait(&bars[warp], 0);
         else cp_async_wait_all();
     }
 
@@ -503,13 +525,27 @@ cudaError_t launch_ptmem(const FactorArgs &a) {
     size_t sm = (size_t)4 * SH::PSM * 32 * 4;
     const size_t floor_sm = SH::COLS == 256 ? 80 * 1024 : 120 * 1024;
     if (sm < floor_sm) sm = floor_sm;
-    auto kern = potrf_ptmem_kernel<N, CT, S, TMA, false, FILL>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-    if (e == cudaSuccess) e = apply_carveout(kern, a.carveout);
-    if (e != cudaSuccess) return e;
-    kern<<<grid_for(a.batch, 128), 128, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride,
-                                                         nullptr);
-    return cudaGetLastError();
+    constexpr int K = S - SH::CS;
+    PtmemMaps<K> maps{};
+    auto go = [&](auto kern) -> cudaError_t {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+        if (e == cudaSuccess) e = apply_carveout(kern, a.carveout);
+        if (e != cudaSuccess) return e;
+        kern<<<grid_for(a.batch, 128), 128, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride, maps,
+                                                             nullptr);
+        return cudaGetLastError();
+    };
+    // per-thread staging requested (no chunk-32 TMA): the shared-memory panel
+    // columns by 2-D TMA where the layout allows (16-B row stride) and where it
+    // measured ahead of the per-thread cp.async form: n = 32..38 (+1-3%; n = 25
+    // and 40: -1 to -3%, elsewhere within 1%: tuning/sweep_b200_r02_tma2d_ab_*.jsonl)
+    if constexpr (!TMA && SH::PSM > 0 && N >= 32 && N <= 38) {
+        bool tm = true;
+        for (int c = SH::CS; c < S && tm; ++c)
+            tm = tma2d_make_map(&maps.m[c - SH::CS], a.A, a.batch, a.cstride, N * N, N - c);
+        if (tm) return go(potrf_ptmem_kernel<N, CT, S, TMA, false, FILL, true>);
+    }
+    return go(potrf_ptmem_kernel<N, CT, S, TMA, false, FILL, false>);
 }
 
 template <int N, int CT, int S, bool TMA>
@@ -521,7 +557,8 @@ cudaError_t launch_sposv_ptmem(const SolveArgs &a) {
     auto kern = potrf_ptmem_kernel<N, CT, S, TMA, true>;
     const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
-    kern<<<grid_for(a.batch, 128), 128, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride, a.B);
+    const PtmemMaps<S - SH::CS> maps{};
+    kern<<<grid_for(a.batch, 128), 128, sm, a.stream>>>(a.A, a.info, a.nfailed, a.batch, a.cstride, maps, a.B);
     return cudaGetLastError();
 }
 
