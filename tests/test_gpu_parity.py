@@ -362,3 +362,21 @@ def test_rcw_many_groups_per_cta(n, chunk):
             ref = out
         else:
             assert np.array_equal(out.view(np.uint32), ref.view(np.uint32)), t
+
+
+@pytest.mark.parametrize("n,chunk,variant,param", [(32, 64, 5, 16), (36, 0, 5, 20), (38, 160, 5, 24),
+                                                   (40, 0, 14, 2), (48, 64, 14, 0), (51, 96, 14, 1)])
+def test_tma2d_staging_bitwise_equal_to_cp_async(monkeypatch, n, chunk, variant, param):
+    """Runtime-chunk staging by 2-D tensor TMA (PTMEM n = 32..38, RCWP n <= 51)
+    and the per-thread cp.async form (BSPOTRF_TMA2D=0) give the same bits, and
+    both pass the oracle, with failures and a partial last group."""
+    batch = 7 * 32 + 20 if chunk == 0 else 7 * 32 + 19
+    canon, inter = make_batch(n, batch, chunk, kind="als", seed=n, fail_seed=2018, fail_period=9)
+    tune = dict(variant=variant, threads_per_block=128 if variant == 5 else 256, param=param,
+                staging=2 if variant == 5 else 0)
+    out1, info1, cnt1 = run_gpu(n, batch, chunk, inter, tune=tune)
+    monkeypatch.setenv("BSPOTRF_TMA2D", "0")
+    out0, info0, cnt0 = run_gpu(n, batch, chunk, inter, tune=tune)
+    assert np.array_equal(out1.view(np.uint32), out0.view(np.uint32))
+    assert np.array_equal(info1, info0) and cnt1 == cnt0
+    assert_parity(n, batch, chunk, canon, inter, out1, info1, cnt1)
