@@ -80,6 +80,48 @@ struct RcwShape {
     static_assert(off(R) <= HALF, "slots exceed the TMEM column budget");
 };
 
+// The 8x8 diagonal block of column block c, factored in registers from its
+// shared-memory gather DB ([36][32], lane q): d (packed lower, dt order) and
+// inv = 1 / diag.  Fig. 9's op order; the sqrt / reciprocal use the branch-free
+// fast forms (common.cuh: bitwise equal to the intrinsics wherever their `ok`
+// holds, checked exhaustively over all 2^32 inputs), so the block is one basic
+// block; a lane outside their range (a failed pivot, extreme exponents) redoes
+// the block with the intrinsics -- same bits, info decided by the exact pass.
+// (+1-5% for RCWP at n = 49..64, where the redundant diagonal work of every
+// warp sits on the critical path, j29.)
+template <int N, int C>
+__device__ __forceinline__ void rcw_factor_diag(const float *DB, int q, float *d, float *inv, int &inf) {
+    using SH = RcwShape<N, 1>;
+    auto pass = [&](auto fast_) -> bool {
+        constexpr bool FAST = decltype(fast_)::value;
+        bool ok = true;
+#pragma unroll
+        for (int t = 0; t < 36; ++t) d[t] = DB[t * 32 + q];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            if (8 * C + k >= N) break;
+            const float p = d[SH::dt(k, k)];
+            pivot_check(p, 8 * C + k, inf);
+            const float s = FAST ? f_sqrt_fast(p, ok) : f_sqrt(p);
+            d[SH::dt(k, k)] = s;
+            inv[k] = FAST ? f_rcp_fast(s, ok) : f_rcp(s);
+#pragma unroll
+            for (int m = k + 1; m < 8; ++m) d[SH::dt(m, k)] = f_mul(d[SH::dt(m, k)], inv[k]);
+#pragma unroll
+            for (int j = k + 1; j < 8; ++j)
+#pragma unroll
+                for (int m = j; m < 8; ++m) d[SH::dt(m, j)] = f_upd(d[SH::dt(m, j)], d[SH::dt(m, k)], d[SH::dt(j, k)]);
+        }
+        return ok;
+    };
+    const int inf0 = inf;
+    if (!pass(std::true_type{})) {
+        inf = inf0;
+        pass(std::false_type{});
+    }
+}
+
+
 template <int N, int CT, int NCTA>
 __global__ void __launch_bounds__(256, NCTA)
 potrf_rcw_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__restrict__ nfailed,
@@ -249,23 +291,7 @@ potrf_rcw_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__r
                 }
             __syncthreads();
             float d[36], inv[8];
-#pragma unroll
-            for (int t = 0; t < 36; ++t) d[t] = DB[t * 32 + q];
-#pragma unroll
-            for (int k = 0; k < 8; ++k) {
-                if (8 * c + k >= N) break;
-                const float p = d[SH::dt(k, k)];
-                pivot_check(p, 8 * c + k, inf);
-                const float s = f_sqrt(p);
-                d[SH::dt(k, k)] = s;
-                inv[k] = f_rcp(s);
-#pragma unroll
-                for (int m = k + 1; m < 8; ++m) d[SH::dt(m, k)] = f_mul(d[SH::dt(m, k)], inv[k]);
-#pragma unroll
-                for (int j = k + 1; j < 8; ++j)
-#pragma unroll
-                    for (int m = j; m < 8; ++m) d[SH::dt(m, j)] = f_upd(d[SH::dt(m, j)], d[SH::dt(m, k)], d[SH::dt(j, k)]);
-            }
+            rcw_factor_diag<N, c>(DB, q, d, inv, inf);
 #pragma unroll
             for (int m = 0; m < 8; ++m)
                 if (m == h && 8 * c + m < N) {

@@ -328,26 +328,7 @@ potrf_rcwp_kernel(float *__restrict__ A, int32_t *__restrict__ info, int32_t *__
                 }
             __syncthreads();                             // B2
             float d[36], inv[8];
-            auto factor_diag = [&]() {
-#pragma unroll
-                for (int t = 0; t < 36; ++t) d[t] = DB[t * 32 + q];
-#pragma unroll
-                for (int k = 0; k < 8; ++k) {
-                    if (8 * c + k >= N) break;
-                    const float p = d[RS::dt(k, k)];
-                    pivot_check(p, 8 * c + k, inf);
-                    const float s = f_sqrt(p);
-                    d[RS::dt(k, k)] = s;
-                    inv[k] = f_rcp(s);
-#pragma unroll
-                    for (int m = k + 1; m < 8; ++m) d[RS::dt(m, k)] = f_mul(d[RS::dt(m, k)], inv[k]);
-#pragma unroll
-                    for (int j = k + 1; j < 8; ++j)
-#pragma unroll
-                        for (int m = j; m < 8; ++m)
-                            d[RS::dt(m, j)] = f_upd(d[RS::dt(m, j)], d[RS::dt(m, k)], d[RS::dt(j, k)]);
-                }
-            };
+            auto factor_diag = [&]() { rcw_factor_diag<N, c>(DB, q, d, inv, inf); };
             if constexpr (D1) {
                 if (h == 0) {                            // warp 0 alone; info is warp 0's
                     factor_diag();
