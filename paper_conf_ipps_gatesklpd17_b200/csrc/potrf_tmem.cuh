@@ -316,9 +316,9 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
         for (int k = 0; k < NB; ++k) {
             const float d = dg[k + k * NB];
             pivot_check(d, CB * NB + k, inf);
-            const float s = f_sqrt(d);
+            const float s = f_sqrt_pos(d);
             dg[k + k * NB] = s;
-            const float inv = f_rcp(s);
+            const float inv = f_rcp_pos(s);
 #pragma unroll
             for (int i = k + 1; i < NB; ++i) dg[i + k * NB] = f_mul(dg[i + k * NB], inv);
 #pragma unroll
@@ -329,7 +329,7 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
         put_tile(CB, dg, cb_, TRUE_{});
         float rinv[NB];
 #pragma unroll
-        for (int k = 0; k < NB; ++k) rinv[k] = f_rcp(dg[k + k * NB]);
+        for (int k = 0; k < NB; ++k) rinv[k] = f_rcp_pos(dg[k + k * NB]);
         float xcb[NB];                                  // forward substitution, this block
         if constexpr (SOLVE) {
 #pragma unroll
@@ -440,9 +440,9 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
         constexpr int k = BSP_CI(k_);
         const float d = r[tri<NT>(k, k)];
         pivot_check(d, k + S, inf);
-        const float s = f_sqrt(d);
+        const float s = f_sqrt_pos(d);
         r[tri<NT>(k, k)] = s;
-        const float inv = f_rcp(s);
+        const float inv = f_rcp_pos(s);
 #pragma unroll
         for (int m = k + 1; m < NT; ++m) r[tri<NT>(m, k)] = f_mul(r[tri<NT>(m, k)], inv);
 #pragma unroll
@@ -468,7 +468,7 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
             float sacc = X[(S + i) * 32];
 #pragma unroll
             for (int j = i + 1; j < NT; ++j) sacc = f_upd(sacc, r[tri<NT>(j, i)], X[(S + j) * 32]);
-            X[(S + i) * 32] = f_mul(sacc, f_rcp(r[tri<NT>(i, i)]));
+            X[(S + i) * 32] = f_mul(sacc, f_rcp_pos(r[tri<NT>(i, i)]));
         });
         // ... panel rows i = S-1..0: column i of L from TMEM tiles / shared memory
 #pragma unroll 1
@@ -496,7 +496,7 @@ potrf_ptmem_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                     if (j > i && j < N) sacc = f_upd(sacc, l[q], X[j * 32]);
                 }
             }
-            X[i * 32] = f_mul(sacc, f_rcp(lii));
+            X[i * 32] = f_mul(sacc, f_rcp_pos(lii));
         }
         if (active && inf == 0) {                       // SPOSV: failed matrices keep B
             const RectAddr<N, CT> ba(Bx, g, cs, 1);

@@ -23,6 +23,13 @@ __global__ void check(unsigned long long *bad, unsigned long long *slow) {
         const bool posnorm = x >= 1.17549435e-38f && x <= 3.40282347e38f;
         if (posnorm && !ok1) ++s[0];
         if (posnorm && !ok2) ++s[1];
+        // the full-range positive forms (f_sqrt_pos / f_rcp_pos): every positive
+        // finite x, and the reciprocal of its root
+        if (i >= 1 && i <= 0x7f7fffffu) {
+            const float r = __fsqrt_rn(x);
+            if (__float_as_uint(bsp::f_sqrt_pos(x)) != __float_as_uint(r)) ++b[0];
+            if (__float_as_uint(bsp::f_rcp_pos(r)) != __float_as_uint(__frcp_rn(r))) ++b[1];
+        }
     }
     atomicAdd(&bad[0], b[0]); atomicAdd(&bad[1], b[1]);
     atomicAdd(&slow[0], s[0]); atomicAdd(&slow[1], s[1]);
