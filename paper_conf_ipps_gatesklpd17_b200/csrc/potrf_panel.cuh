@@ -144,9 +144,9 @@ potrf_panel_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                 for (int k = 0; k < NB; ++k) {
                     const float d = acc[k + k * NB];
                     pivot_check(d, cb * NB + k, inf);
-                    const float s = f_sqrt(d);
+                    const float s = f_sqrt_pos(d);
                     acc[k + k * NB] = s;
-                    const float inv = f_rcp(s);
+                    const float inv = f_rcp_pos(s);
 #pragma unroll
                     for (int i = k + 1; i < NB; ++i) acc[i + k * NB] = f_mul(acc[i + k * NB], inv);
 #pragma unroll
@@ -164,7 +164,7 @@ potrf_panel_kernel(float *__restrict__ A, int32_t *__restrict__ info,
                     for (int i = j; i < NB; ++i) l[i + j * NB] = P[(cbase[j] + cb * NB + i) * BL];
 #pragma unroll
                 for (int k = 0; k < NB; ++k) {
-                    const float inv = f_rcp(l[k + k * NB]);
+                    const float inv = f_rcp_pos(l[k + k * NB]);
 #pragma unroll
                     for (int i = 0; i < NB; ++i) acc[i + k * NB] = f_mul(acc[i + k * NB], inv);
 #pragma unroll
@@ -206,9 +206,9 @@ potrf_panel_kernel(float *__restrict__ A, int32_t *__restrict__ info,
         constexpr int k = BSP_CI(k_);
         const float d = r[tri<NT>(k, k)];
         pivot_check(d, k + S, inf);
-        const float s = f_sqrt(d);
+        const float s = f_sqrt_pos(d);
         r[tri<NT>(k, k)] = s;
-        const float inv = f_rcp(s);
+        const float inv = f_rcp_pos(s);
 #pragma unroll
         for (int m = k + 1; m < NT; ++m) r[tri<NT>(m, k)] = f_mul(r[tri<NT>(m, k)], inv);
 #pragma unroll
